@@ -1,0 +1,197 @@
+/*
+ * eggsync.h -- C ABI of the B200-native EGG-SynC synchronization update.
+ *
+ * Paper: J. R. Jorgensen, I. Assent, "EGG-SynC: Exact GPU-parallelized
+ * Grid-based Clustering by Synchronization", EDBT 2023.  Citations "L<n>"
+ * are lines of that paper's text with the section / equation /
+ * algorithm they fall in.
+ *
+ * Problem statement (L66-L70 §3, Def 4.1): given D in [0,1]^{n x d}
+ * and a radius eps, iterate the Kuramoto update (Eq.1)
+ *     p_i <- p_i + 1/|N_eps(p)| * sum_{q in N_eps(p)} sin(q_i - p_i),
+ *     N_eps(p) = {q : ||p - q|| <= eps}  (p itself included, L66)
+ * synchronously until the synchronization criterion (Def 4.2)
+ * holds, then return the clusters: the non-empty grid cells of width
+ * eps/(2 sqrt d) (gatherCluster, L256; cell width L252).
+ *
+ * Conventions shared by every entry point
+ *  - All functions have C linkage, are reentrant with respect to distinct
+ *    buffers, and never throw across the ABI.
+ *  - Ownership: the caller owns every buffer passed in.  The library
+ *    allocates its device workspace per call (or per context), reuses it
+ *    across iterations (as the paper does, L195) and frees it before
+ *    returning (or in eggsync_ctx_destroy).
+ *  - Validation happens before any output is written: on EGGSYNC_EINVAL or
+ *    EGGSYNC_EDOMAIN every output buffer is left untouched.  After
+ *    EGGSYNC_ENOMEM / EGGSYNC_ECUDA outputs are unspecified.
+ *  - eps is used exactly as the given float; every derived constant
+ *    (eps^2, c_w, 1/c_w, w, delta) is computed in fp64 from (double)eps.
+ *  - Arithmetic: coordinates are float32; neighbour sums are accumulated in
+ *    fp32 chunks flushed into fp64; cell / subtree summaries are exact
+ *    64-bit fixed-point sums of fp64 sin/cos; the update epilogue is fp64.
+ *    The eps-predicate is decided in fp32 with a proven error band; pairs
+ *    inside the band are re-decided in fp64 exactly as sum_i (q_i - p_i)^2
+ *    <= eps^2 (dimension order, no FMA).
+ *  - There is no CPU fallback: without a usable CUDA device every compute
+ *    entry point returns EGGSYNC_ECUDA.
+ */
+#ifndef EGGSYNC_H
+#define EGGSYNC_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define EGGSYNC_OK 0
+#define EGGSYNC_NOT_CONVERGED 1 /* max_iters reached: outputs hold the last state, labels = its cells */
+#define EGGSYNC_EINVAL (-1)     /* NULL pointer, n < 1 or n > INT32_MAX, d < 1 or d > EGGSYNC_MAX_D,
+                                   eps not finite or <= 0, grid too fine (d*ceil(log2 w) > 512 bits) */
+#define EGGSYNC_EDOMAIN (-2)    /* a coordinate is NaN/Inf or outside [0,1] (L70, L290, L354) */
+#define EGGSYNC_ENOMEM (-3)     /* device allocation failed */
+#define EGGSYNC_ECUDA (-4)      /* CUDA error or no device; details in eggsync_last_error() */
+#define EGGSYNC_ENCCL (-5)      /* reserved: collective failure (multi-GPU driver) */
+
+#define EGGSYNC_MAX_D 32
+
+/* termination modes (ambiguity register R1/F3 in DESIGN.md) */
+#define EGGSYNC_TERM_GRID 0 /* first term via |cell(p)| == |N_eps(p)| (Alg 3 l.14-15 L248, L252) */
+
+/*
+ * Per-stage timings of the last call, mirroring the columns of Table 1
+ * (L364-371): allocating, build structure, update, extra check,
+ * clustering, free.  Seconds, measured with CUDA events on the call's
+ * stream.  Work counters are summed over iterations.
+ */
+typedef struct eggsync_stats {
+  double t_alloc, t_build, t_update, t_extra_check, t_cluster, t_free, t_transfer;
+  int32_t iters;
+  int32_t n_cells_first, n_cells_last;
+  int32_t sort_skipped; /* iterations whose keys were already sorted */
+  int64_t device_bytes; /* workspace high-water mark */
+} eggsync_stats;
+
+typedef struct eggsync_opts {
+  int32_t struct_size;     /* sizeof(eggsync_opts); ABI versioning */
+  int32_t max_iters;       /* default 10000 (L306: "a maximum number of iterations could be used") */
+  int32_t device;          /* CUDA ordinal; -1 = current device */
+  int32_t device_pointers; /* 1: points / labels / coords_out / nbr_count_out are device pointers */
+  void *stream;            /* cudaStream_t to run on; NULL = library-owned stream */
+  int32_t term_mode;       /* EGGSYNC_TERM_GRID (only mode implemented) */
+  float *coords_out;       /* optional n*d row-major final coordinates (original point order) */
+  int32_t *nbr_count_out;  /* optional, step only: |N_eps(p)| on D^t, original order */
+  eggsync_stats *stats;    /* optional */
+} eggsync_opts;
+
+/* Fill *o with the defaults above (struct_size set). */
+void eggsync_default_opts(eggsync_opts *o);
+
+/*
+ * eggsync_cluster -- EGG-SynC(D, eps) (Algorithm 4).
+ *   points     : n*d float32, row-major, values in [0,1]; HOST memory
+ *   n, d, eps  : sizes and the neighbourhood radius (L66)
+ *   labels_out : n int32 (host); cluster id per point, clusters numbered
+ *                0..k-1 by their smallest point index (canonical)
+ *   iters_out  : number of Eq.1 updates applied (Alg 4's t at exit)
+ * Returns EGGSYNC_OK, EGGSYNC_NOT_CONVERGED, or a negative error code.
+ */
+int eggsync_cluster(const float *points, int64_t n, int32_t d, float eps, int32_t *labels_out,
+                    int32_t *iters_out);
+
+/* As eggsync_cluster with options (device pointers, stream, stats, coords_out, max_iters). */
+int eggsync_cluster_ex(const float *points, int64_t n, int32_t d, float eps, const eggsync_opts *opts,
+                       int32_t *labels_out, int32_t *iters_out);
+
+/*
+ * eggsync_step -- one pass of the loop body of Algorithm 4 on the caller's
+ * state (for testing / resuming):
+ *   points     : in D^t, out D^{t+1} (one synchronous Eq.1 update), n*d row-major float32, host
+ *   synced_out : 1 iff the synchronization criterion (Def 4.2 in its grid
+ *                form: first term |cell(p)| == |N_eps(p)| for all p, L252;
+ *                second term L108-110, L254) holds on D^t, else 0
+ */
+int eggsync_step(float *points, int64_t n, int32_t d, float eps, int32_t *synced_out);
+
+/*
+ * As eggsync_step with options.  first_term_out / second_term_out may be NULL;
+ * second_term_out is -1 when the first term fails (the paper only checks the
+ * second term when the first holds, Alg 4 l.9-10 L273-275).
+ */
+int eggsync_step_ex(float *points, int64_t n, int32_t d, float eps, const eggsync_opts *opts,
+                    int32_t *first_term_out, int32_t *second_term_out);
+
+/* Thread-local message describing the last non-OK return of this thread. */
+const char *eggsync_last_error(void);
+
+/* Library version string. */
+const char *eggsync_version(void);
+
+/* ------------------------------------------------------------------------
+ * Context (phase) API -- device-resident state for the multi-GPU driver and
+ * for device-timed benchmarking.  Every pointer below is DEVICE memory on
+ * the context's device; every call is asynchronous on the context's stream
+ * except where a host output is written (then the call synchronises).
+ *
+ * Multi-GPU scheme: each rank holds all n points,
+ * builds the identical grid (deterministic), updates only its contiguous
+ * range [lo, hi) of the sorted order, and the caller all-gathers the owned
+ * ranges (NCCL via torch.distributed) between eggsync_ctx_update and
+ * eggsync_ctx_advance.  The termination flags are reduced with MIN.
+ * ---------------------------------------------------------------------- */
+typedef struct eggsync_ctx eggsync_ctx;
+
+/* Create a context for n points of d dims; stream may be NULL (library-owned). */
+int eggsync_ctx_create(int64_t n, int32_t d, float eps, int32_t device, void *stream, eggsync_ctx **out);
+void eggsync_ctx_destroy(eggsync_ctx *ctx);
+
+/* Load D^0: points is n*d row-major float32 (device pointer if on_device, else host). Validates [0,1]. */
+int eggsync_ctx_load(eggsync_ctx *ctx, const float *points, int32_t on_device);
+
+/* Build structure for the current state: cell keys, radix sort, cell offsets,
+ * cell summaries, subtree hierarchy (L139-220 §4.2, Eq.5-6).
+ * n_cells_out (host, may be NULL) receives the number of non-empty cells. */
+int eggsync_ctx_build(eggsync_ctx *ctx, int32_t *n_cells_out);
+
+/* EGG-update (Alg 3) of the sorted positions [lo, hi) into the next-state
+ * buffer, plus the first-term flag of those points (device int32, AND-reduced). */
+int eggsync_ctx_update(eggsync_ctx *ctx, int64_t lo, int64_t hi);
+
+/* Second term of Def 4.2 (L108-110, L254) for sorted positions [lo, hi) on the current state. */
+int eggsync_ctx_second_term(eggsync_ctx *ctx, int64_t lo, int64_t hi);
+
+/* Read the flags: first = AND over updated points since the last build; second
+ * = AND over checked points (-1 if never checked since the last build).  Synchronises. */
+int eggsync_ctx_flags(eggsync_ctx *ctx, int32_t *first_out, int32_t *second_out);
+
+/* Device pointers of the state: cur = D^t (SoA [d][n], sorted order), next = D^{t+1}
+ * being written by eggsync_ctx_update. */
+float *eggsync_ctx_cur_coords(eggsync_ctx *ctx);
+float *eggsync_ctx_next_coords(eggsync_ctx *ctx);
+
+/* Pack next-state columns [lo, lo+cnt) into buf (device, [d][cnt]); unpack a
+ * gathered buffer ([ranks][d][cnt], rank r owning [r*cnt, min(n,(r+1)*cnt)))
+ * into the next-state buffer.  Used around an NCCL all-gather. */
+int eggsync_ctx_pack(eggsync_ctx *ctx, int64_t lo, int64_t cnt, float *buf);
+int eggsync_ctx_unpack(eggsync_ctx *ctx, const float *gathered, int32_t ranks, int64_t cnt);
+
+/* Make D^{t+1} the current state (t <- t+1). */
+int eggsync_ctx_advance(eggsync_ctx *ctx);
+
+/* Labels of the current state's cells (gatherCluster L256), canonical, written
+ * to labels (n int32, device if on_device else host), original point order. */
+int eggsync_ctx_labels(eggsync_ctx *ctx, int32_t *labels, int32_t on_device);
+
+/* Current coordinates in original point order, n*d row-major (device if on_device). */
+int eggsync_ctx_coords(eggsync_ctx *ctx, float *coords, int32_t on_device);
+
+/* Run the whole loop (Alg 4) on the context's state; iters_out (host). */
+int eggsync_ctx_run(eggsync_ctx *ctx, int32_t max_iters, int32_t *iters_out);
+
+/* Stream of the context (cudaStream_t). */
+void *eggsync_ctx_stream(eggsync_ctx *ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* EGGSYNC_H */

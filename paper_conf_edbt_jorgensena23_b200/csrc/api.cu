@@ -1,0 +1,631 @@
+// api.cu -- C ABI (include/eggsync.h), workspace and the host loop of
+// Algorithm 4.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstdarg>
+#include <cstring>
+#include <string>
+
+#include "common.cuh"
+
+namespace egg {
+
+template <int D>
+int run_update(Workspace&, int64_t, int64_t, int32_t*);
+template <int D>
+int run_second_term(Workspace&, int64_t, int64_t);
+size_t cub_temp_bytes(int64_t n);
+
+static thread_local std::string g_err;
+
+void set_error(const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+}
+
+bool make_consts(int64_t n, int d, float eps, Consts* c, std::string* why) {
+  if (!(eps > 0.f) || !std::isfinite(eps)) {
+    *why = "eps must be finite and > 0";
+    return false;
+  }
+  c->n = n;
+  c->d = d;
+  c->e = (double)eps;
+  c->e2 = c->e * c->e;
+  c->cw = c->e / (2.0 * std::sqrt((double)d));  // L252: cell diagonal = eps/2
+  c->inv_cw = 1.0 / c->cw;
+  const double wd = std::ceil(1.0 / c->cw);     // Eq.4
+  if (wd > 2147483647.0) {
+    *why = "grid too fine (ceil(1/c_w) > 2^31)";
+    return false;
+  }
+  c->w = (int64_t)wd;
+  int bits = 0;
+  while ((int64_t(1) << bits) < c->w) ++bits;
+  c->bits = std::max(bits, 1);
+  c->keybits = d * c->bits;
+  c->nw = (c->keybits + 63) / 64;
+  if (c->nw > kMaxKeyWords) {
+    *why = "grid too fine: d*ceil(log2 w) > 512 key bits";
+    return false;
+  }
+  c->delta = c->e - c->e * std::sqrt(15.0 / 16.0) + c->e / 2.0 - std::sin(c->e / 2.0);  // L110
+  c->ed = c->e + c->delta;
+  c->ed2 = c->ed * c->ed;
+  c->ef = eps;
+  c->e2f = (float)c->e2;
+  c->edf = (float)c->ed;
+  c->ed2f = (float)c->ed2;
+  c->rel = (float)(4 * d + 16) * kU;
+  return true;
+}
+
+// ------------------------------------------------------------------ workspace
+int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
+  std::string why;
+  if (!make_consts(n_, d_, eps, &k, &why)) {
+    set_error("%s", why.c_str());
+    return EGGSYNC_EINVAL;
+  }
+  n = n_;
+  d = d_;
+  cap = n_;
+  device = dev;
+  const int nw = k.nw;
+  const int CREC = ceil4(3 * d + 3), BS = ceil4(2 * d);
+  cub_bytes = cub_temp_bytes(n);
+  struct Item {
+    void** p;
+    size_t bytes;
+  };
+  Item items[] = {
+      {(void**)&xs[0], sizeof(float) * d * n},
+      {(void**)&xs[1], sizeof(float) * d * n},
+      {(void**)&orig[0], sizeof(uint32_t) * n},
+      {(void**)&orig[1], sizeof(uint32_t) * n},
+      {(void**)&keys, sizeof(uint64_t) * nw * n},
+      {(void**)&keys_tmp, sizeof(uint64_t) * nw * n},
+      {(void**)&kb[0], sizeof(uint64_t) * n},
+      {(void**)&kb[1], sizeof(uint64_t) * n},
+      {(void**)&pb[0], sizeof(uint32_t) * n},
+      {(void**)&pb[1], sizeof(uint32_t) * n},
+      {(void**)&cub_tmp, cub_bytes},
+      {(void**)&sn, sizeof(float) * d * n},
+      {(void**)&cs, sizeof(float) * d * n},
+      {(void**)&cell_of, sizeof(int32_t) * n},
+      {(void**)&iscan, sizeof(int32_t) * n},
+      {(void**)&cell_start, sizeof(int32_t) * (cap + 1)},
+      {(void**)&c_fix, sizeof(uint64_t) * 2 * d * cap},
+      {(void**)&c_lo, sizeof(uint32_t) * d * cap},
+      {(void**)&c_hi, sizeof(uint32_t) * d * cap},
+      {(void**)&c_cnt, sizeof(int32_t) * cap},
+      {(void**)&c_rec, sizeof(float) * CREC * cap},
+      {(void**)&c_key, sizeof(uint64_t) * nw * cap},
+      {(void**)&t_meta, sizeof(int4) * cap},
+      {(void**)&t_parent, sizeof(int32_t) * cap},
+      {(void**)&l_parent, sizeof(int32_t) * cap},
+      {(void**)&t_visit, sizeof(uint32_t) * cap},
+      {(void**)&t_fix, sizeof(uint64_t) * 2 * d * cap},
+      {(void**)&t_lo, sizeof(uint32_t) * d * cap},
+      {(void**)&t_hi, sizeof(uint32_t) * d * cap},
+      {(void**)&t_cnt, sizeof(int32_t) * cap},
+      {(void**)&t_box, sizeof(float) * BS * cap},
+      {(void**)&t_sum, sizeof(float) * BS * cap},
+      {(void**)&flags, sizeof(int32_t) * 8},
+      {(void**)&io, sizeof(float) * d * n},
+      {(void**)&i_lab, sizeof(int32_t) * n},
+      {(void**)&c_minorig, sizeof(uint32_t) * cap},
+      {(void**)&nbr, sizeof(int32_t) * n},
+      {(void**)&lab_final, sizeof(int32_t) * n},
+  };
+  size_t total = 0;
+  for (auto& it : items) total += (it.bytes + 255) & ~size_t(255);
+  char* base = nullptr;
+  cudaError_t e = cudaMalloc((void**)&base, total);
+  if (e != cudaSuccess) {
+    set_error("cudaMalloc(%zu bytes) failed: %s", total, cudaGetErrorString(e));
+    cudaGetLastError();
+    return e == cudaErrorMemoryAllocation ? EGGSYNC_ENOMEM : EGGSYNC_ECUDA;
+  }
+  arena = base;
+  size_t off = 0;
+  for (auto& it : items) {
+    *it.p = base + off;
+    off += (it.bytes + 255) & ~size_t(255);
+  }
+  bytes = (int64_t)total;
+  EGG_CUDA(cudaMallocHost((void**)&h_flags, 16 * sizeof(int32_t)));
+  if (st) {
+    stream = st;
+    own_stream = false;
+  } else {
+    EGG_CUDA(cudaStreamCreateWithFlags(&stream, cudaStreamNonBlocking));
+    own_stream = true;
+  }
+  for (auto& v : ev) EGG_CUDA(cudaEventCreate(&v));
+  ev_ok = true;
+  EGG_CUDA(cudaMemsetAsync(flags, 0, 8 * sizeof(int32_t), stream));
+  return EGGSYNC_OK;
+}
+
+void Workspace::release() {
+  if (arena) cudaFree(arena);
+  arena = nullptr;
+  if (h_flags) cudaFreeHost(h_flags);
+  h_flags = nullptr;
+  if (own_stream && stream) cudaStreamDestroy(stream);
+  stream = nullptr;
+  own_stream = false;
+  if (ev_ok)
+    for (auto& v : ev) cudaEventDestroy(v);
+  ev_ok = false;
+}
+
+#define EGG_CASE_D(Dv, FN, ...) \
+  case Dv:                      \
+    return FN<Dv>(__VA_ARGS__);
+#define EGG_DISPATCH(d, FN, ...)                                                                        \
+  switch (d) {                                                                                          \
+    EGG_CASE_D(1, FN, __VA_ARGS__) EGG_CASE_D(2, FN, __VA_ARGS__) EGG_CASE_D(3, FN, __VA_ARGS__)        \
+    EGG_CASE_D(4, FN, __VA_ARGS__) EGG_CASE_D(5, FN, __VA_ARGS__) EGG_CASE_D(6, FN, __VA_ARGS__)        \
+    EGG_CASE_D(7, FN, __VA_ARGS__) EGG_CASE_D(8, FN, __VA_ARGS__) EGG_CASE_D(9, FN, __VA_ARGS__)        \
+    EGG_CASE_D(10, FN, __VA_ARGS__) EGG_CASE_D(11, FN, __VA_ARGS__) EGG_CASE_D(12, FN, __VA_ARGS__)     \
+    EGG_CASE_D(13, FN, __VA_ARGS__) EGG_CASE_D(14, FN, __VA_ARGS__) EGG_CASE_D(15, FN, __VA_ARGS__)     \
+    EGG_CASE_D(16, FN, __VA_ARGS__) EGG_CASE_D(17, FN, __VA_ARGS__) EGG_CASE_D(18, FN, __VA_ARGS__)     \
+    EGG_CASE_D(19, FN, __VA_ARGS__) EGG_CASE_D(20, FN, __VA_ARGS__) EGG_CASE_D(21, FN, __VA_ARGS__)     \
+    EGG_CASE_D(22, FN, __VA_ARGS__) EGG_CASE_D(23, FN, __VA_ARGS__) EGG_CASE_D(24, FN, __VA_ARGS__)     \
+    EGG_CASE_D(25, FN, __VA_ARGS__) EGG_CASE_D(26, FN, __VA_ARGS__) EGG_CASE_D(27, FN, __VA_ARGS__)     \
+    EGG_CASE_D(28, FN, __VA_ARGS__) EGG_CASE_D(29, FN, __VA_ARGS__) EGG_CASE_D(30, FN, __VA_ARGS__)     \
+    EGG_CASE_D(31, FN, __VA_ARGS__) EGG_CASE_D(32, FN, __VA_ARGS__)                                    \
+    default:                                                                                            \
+      set_error("unsupported d=%d", d);                                                                 \
+      return EGGSYNC_EINVAL;                                                                            \
+  }
+
+int stage_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
+  EGG_DISPATCH(ws.d, run_update, ws, lo, hi, nbr);
+}
+int stage_second_term(Workspace& ws, int64_t lo, int64_t hi) {
+  EGG_DISPATCH(ws.d, run_second_term, ws, lo, hi);
+}
+
+__global__ void k_set_flags(int32_t* f, int32_t a, int32_t b) {
+  f[0] = a;
+  f[1] = b;
+}
+__global__ void k_pack(const float* __restrict__ xs, int64_t n, int d, int64_t lo, int64_t cnt,
+                       float* __restrict__ buf) {
+  int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= cnt * d) return;
+  int i = (int)(t / cnt);
+  int64_t k = t - (int64_t)i * cnt;
+  int64_t pos = lo + k;
+  buf[t] = pos < n ? xs[(int64_t)i * n + pos] : 0.f;
+}
+__global__ void k_unpack(const float* __restrict__ g, int64_t n, int d, int32_t ranks, int64_t cnt,
+                         float* __restrict__ xs) {
+  int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= (int64_t)ranks * d * cnt) return;
+  int64_t per_rank = (int64_t)d * cnt;
+  int64_t r = t / per_rank;
+  int64_t rem = t - r * per_rank;
+  int i = (int)(rem / cnt);
+  int64_t k = rem - (int64_t)i * cnt;
+  int64_t pos = r * cnt + k;
+  if (pos < n) xs[(int64_t)i * n + pos] = g[t];
+}
+
+static int read_flags(Workspace& ws, int32_t* f1, int32_t* f2, int32_t* err) {
+  EGG_CUDA(cudaMemcpyAsync(ws.h_flags, ws.flags, 4 * sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
+  EGG_CUDA(cudaStreamSynchronize(ws.stream));
+  if (f1) *f1 = ws.h_flags[0];
+  if (f2) *f2 = ws.h_flags[1];
+  if (err) *err = ws.h_flags[3];
+  if (ws.h_flags[3]) {
+    set_error("traversal stack overflow (internal error)");
+    return EGGSYNC_ECUDA;
+  }
+  return EGGSYNC_OK;
+}
+
+static double ev_ms(cudaEvent_t a, cudaEvent_t b) {
+  float ms = 0.f;
+  cudaEventElapsedTime(&ms, a, b);
+  return ms * 1e-3;
+}
+
+// One pass of Alg 4's loop body: build, update, first term, (second term).
+// Returns synced through *synced; labels of the verified state into lab (device) when synced.
+static int iterate(Workspace& ws, int32_t* synced, int32_t* f1o, int32_t* f2o, int32_t* nbr_sorted,
+                   eggsync_stats* stats) {
+  if (stats) EGG_CUDA(cudaEventRecord(ws.ev[0], ws.stream));
+  if (!ws.built) EGG_TRY(stage_build(ws));
+  if (stats) EGG_CUDA(cudaEventRecord(ws.ev[1], ws.stream));
+  k_set_flags<<<1, 1, 0, ws.stream>>>(ws.flags, 1, 1);
+  EGG_CUDA(cudaGetLastError());
+  EGG_TRY(stage_update(ws, 0, ws.n, nbr_sorted));
+  if (stats) EGG_CUDA(cudaEventRecord(ws.ev[2], ws.stream));
+  int32_t f1 = 0, f2 = -1, err = 0;
+  EGG_TRY(read_flags(ws, &f1, nullptr, &err));
+  if (stats) {
+    stats->t_build += ev_ms(ws.ev[0], ws.ev[1]);
+    stats->t_update += ev_ms(ws.ev[1], ws.ev[2]);
+  }
+  if (f1) {
+    if (stats) EGG_CUDA(cudaEventRecord(ws.ev[3], ws.stream));
+    EGG_TRY(stage_second_term(ws, 0, ws.n));
+    if (stats) EGG_CUDA(cudaEventRecord(ws.ev[4], ws.stream));
+    EGG_TRY(read_flags(ws, nullptr, &f2, &err));
+    if (stats) stats->t_extra_check += ev_ms(ws.ev[3], ws.ev[4]);
+  }
+  *synced = (f1 && f2 == 1) ? 1 : 0;
+  if (f1o) *f1o = f1;
+  if (f2o) *f2o = f1 ? f2 : -1;
+  return EGGSYNC_OK;
+}
+
+static void advance(Workspace& ws) {
+  ws.xcur ^= 1;
+  ws.built = false;
+}
+
+// Algorithm 4: iterate until the criterion holds on the state the update read
+// (reading R6/R7), labels = cells of that state (gatherCluster, L256).
+static int run_loop(Workspace& ws, int32_t max_iters, int32_t* iters_out, eggsync_stats* stats) {
+  int32_t t = 0, synced = 0;
+  ws.have_final = false;
+  for (;;) {
+    EGG_TRY(iterate(ws, &synced, nullptr, nullptr, nullptr, stats));
+    if (stats) {
+      if (t == 0) stats->n_cells_first = ws.n_cells;
+      stats->n_cells_last = ws.n_cells;
+    }
+    if (synced) {
+      if (stats) EGG_CUDA(cudaEventRecord(ws.ev[5], ws.stream));
+      EGG_TRY(stage_labels(ws, ws.lab_final));
+      if (stats) EGG_CUDA(cudaEventRecord(ws.ev[6], ws.stream));
+      ws.have_final = true;
+    }
+    advance(ws);
+    ++t;
+    if (synced || t >= max_iters) break;
+  }
+  if (!synced) {
+    EGG_TRY(stage_build(ws));
+    EGG_TRY(stage_labels(ws, ws.lab_final));
+    ws.have_final = true;
+  }
+  EGG_CUDA(cudaStreamSynchronize(ws.stream));
+  if (stats && synced) stats->t_cluster += ev_ms(ws.ev[5], ws.ev[6]);
+  if (stats) {
+    stats->iters = t;
+    stats->sort_skipped = ws.sort_skipped;
+  }
+  *iters_out = t;
+  return synced ? EGGSYNC_OK : EGGSYNC_NOT_CONVERGED;
+}
+
+struct DeviceGuard {
+  int prev = -1;
+  bool changed = false;
+  int set(int dev) {
+    if (dev < 0) return EGGSYNC_OK;
+    EGG_CUDA(cudaGetDevice(&prev));
+    if (prev != dev) {
+      EGG_CUDA(cudaSetDevice(dev));
+      changed = true;
+    }
+    return EGGSYNC_OK;
+  }
+  ~DeviceGuard() {
+    if (changed) cudaSetDevice(prev);
+  }
+};
+
+static int validate(const void* points, int64_t n, int32_t d, float eps) {
+  if (!points) {
+    set_error("points is NULL");
+    return EGGSYNC_EINVAL;
+  }
+  if (n < 1 || n > INT32_MAX) {
+    set_error("n=%lld out of range [1, 2^31-1]", (long long)n);
+    return EGGSYNC_EINVAL;
+  }
+  if (d < 1 || d > EGGSYNC_MAX_D) {
+    set_error("d=%d out of range [1, %d]", d, EGGSYNC_MAX_D);
+    return EGGSYNC_EINVAL;
+  }
+  Consts c;
+  std::string why;
+  if (!make_consts(n, d, eps, &c, &why)) {
+    set_error("%s", why.c_str());
+    return EGGSYNC_EINVAL;
+  }
+  return EGGSYNC_OK;
+}
+
+static int check_device() {
+  int cnt = 0;
+  cudaError_t e = cudaGetDeviceCount(&cnt);
+  if (e != cudaSuccess || cnt < 1) {
+    cudaGetLastError();
+    set_error("no CUDA device available (%s); there is no CPU fallback",
+              e != cudaSuccess ? cudaGetErrorString(e) : "0 devices");
+    return EGGSYNC_ECUDA;
+  }
+  return EGGSYNC_OK;
+}
+
+}  // namespace egg
+
+using namespace egg;
+
+struct eggsync_ctx {
+  Workspace ws;
+};
+
+extern "C" {
+
+const char* eggsync_last_error(void) { return g_err.c_str(); }
+const char* eggsync_version(void) { return "eggsync-b200 0.1 (sm_100a)"; }
+
+void eggsync_default_opts(eggsync_opts* o) {
+  if (!o) return;
+  memset(o, 0, sizeof *o);
+  o->struct_size = (int32_t)sizeof(eggsync_opts);
+  o->max_iters = 10000;
+  o->device = -1;
+  o->term_mode = EGGSYNC_TERM_GRID;
+}
+
+static int get_opts(const eggsync_opts* in, eggsync_opts* o) {
+  eggsync_default_opts(o);
+  if (!in) return EGGSYNC_OK;
+  if (in->struct_size != (int32_t)sizeof(eggsync_opts)) {
+    set_error("eggsync_opts.struct_size mismatch (%d != %d)", in->struct_size, (int)sizeof(eggsync_opts));
+    return EGGSYNC_EINVAL;
+  }
+  *o = *in;
+  if (o->max_iters < 1) {
+    set_error("max_iters must be >= 1");
+    return EGGSYNC_EINVAL;
+  }
+  if (o->term_mode != EGGSYNC_TERM_GRID) {
+    set_error("term_mode %d not implemented (only EGGSYNC_TERM_GRID)", o->term_mode);
+    return EGGSYNC_EINVAL;
+  }
+  return EGGSYNC_OK;
+}
+
+int eggsync_cluster_ex(const float* points, int64_t n, int32_t d, float eps, const eggsync_opts* opts,
+                       int32_t* labels_out, int32_t* iters_out) {
+  eggsync_opts o;
+  EGG_TRY(get_opts(opts, &o));
+  EGG_TRY(validate(points, n, d, eps));
+  if (!labels_out || !iters_out) {
+    set_error("labels_out / iters_out is NULL");
+    return EGGSYNC_EINVAL;
+  }
+  EGG_TRY(check_device());
+  DeviceGuard g;
+  EGG_TRY(g.set(o.device));
+  eggsync_stats local{};
+  eggsync_stats* stats = o.stats ? &local : nullptr;
+  auto t0 = std::chrono::steady_clock::now();
+  Workspace ws;
+  EGG_TRY(ws.alloc(n, d, eps, o.device, (cudaStream_t)o.stream));
+  EGG_CUDA(cudaStreamSynchronize(ws.stream));
+  auto t1 = std::chrono::steady_clock::now();
+  if (stats) stats->t_alloc = std::chrono::duration<double>(t1 - t0).count();
+  EGG_TRY(stage_ingest(ws, points, o.device_pointers != 0));
+  auto t2 = std::chrono::steady_clock::now();
+  int32_t iters = 0;
+  int rc = run_loop(ws, o.max_iters, &iters, stats);
+  if (rc < 0) return rc;
+  // outputs
+  auto t3 = std::chrono::steady_clock::now();
+  if (o.device_pointers) {
+    EGG_CUDA(cudaMemcpyAsync(labels_out, ws.lab_final, sizeof(int32_t) * n, cudaMemcpyDeviceToDevice, ws.stream));
+    if (o.coords_out) EGG_TRY(stage_coords(ws, ws.xcur, o.coords_out));
+  } else {
+    EGG_CUDA(cudaMemcpyAsync(labels_out, ws.lab_final, sizeof(int32_t) * n, cudaMemcpyDeviceToHost, ws.stream));
+    if (o.coords_out) {
+      EGG_TRY(stage_coords(ws, ws.xcur, ws.io));
+      EGG_CUDA(cudaMemcpyAsync(o.coords_out, ws.io, sizeof(float) * n * d, cudaMemcpyDeviceToHost, ws.stream));
+    }
+  }
+  EGG_CUDA(cudaStreamSynchronize(ws.stream));
+  auto t4 = std::chrono::steady_clock::now();
+  *iters_out = iters;
+  if (stats) {
+    local.t_transfer = std::chrono::duration<double>(t2 - t1).count() +
+                       std::chrono::duration<double>(t4 - t3).count();
+    local.device_bytes = ws.bytes;
+    ws.release();
+    local.t_free = std::chrono::duration<double>(std::chrono::steady_clock::now() - t4).count();
+    *o.stats = local;
+  }
+  return rc;
+}
+
+int eggsync_cluster(const float* points, int64_t n, int32_t d, float eps, int32_t* labels_out,
+                    int32_t* iters_out) {
+  return eggsync_cluster_ex(points, n, d, eps, nullptr, labels_out, iters_out);
+}
+
+int eggsync_step_ex(float* points, int64_t n, int32_t d, float eps, const eggsync_opts* opts,
+                    int32_t* first_term_out, int32_t* second_term_out) {
+  eggsync_opts o;
+  EGG_TRY(get_opts(opts, &o));
+  EGG_TRY(validate(points, n, d, eps));
+  EGG_TRY(check_device());
+  DeviceGuard g;
+  EGG_TRY(g.set(o.device));
+  Workspace ws;
+  EGG_TRY(ws.alloc(n, d, eps, o.device, (cudaStream_t)o.stream));
+  EGG_TRY(stage_ingest(ws, points, o.device_pointers != 0));
+  int32_t synced = 0, f1 = 0, f2 = -1;
+  EGG_TRY(iterate(ws, &synced, &f1, &f2, o.nbr_count_out ? ws.nbr : nullptr, nullptr));
+  // nbr counts refer to D^t's sorted order -> original order
+  if (o.nbr_count_out) {
+    EGG_TRY(stage_scatter_i32(ws, ws.nbr, ws.i_lab));
+    EGG_CUDA(cudaMemcpyAsync(o.nbr_count_out, ws.i_lab, sizeof(int32_t) * n,
+                             o.device_pointers ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, ws.stream));
+  }
+  advance(ws);
+  if (o.device_pointers) {
+    EGG_TRY(stage_coords(ws, ws.xcur, points));
+  } else {
+    EGG_TRY(stage_coords(ws, ws.xcur, ws.io));
+    EGG_CUDA(cudaMemcpyAsync(points, ws.io, sizeof(float) * n * d, cudaMemcpyDeviceToHost, ws.stream));
+  }
+  EGG_CUDA(cudaStreamSynchronize(ws.stream));
+  if (first_term_out) *first_term_out = f1;
+  if (second_term_out) *second_term_out = f2;
+  return EGGSYNC_OK;
+}
+
+int eggsync_step(float* points, int64_t n, int32_t d, float eps, int32_t* synced_out) {
+  int32_t f1 = 0, f2 = -1;
+  int rc = eggsync_step_ex(points, n, d, eps, nullptr, &f1, &f2);
+  if (rc == EGGSYNC_OK && synced_out) *synced_out = (f1 && f2 == 1) ? 1 : 0;
+  return rc;
+}
+
+// ------------------------------------------------------------------ context
+int eggsync_ctx_create(int64_t n, int32_t d, float eps, int32_t device, void* stream, eggsync_ctx** out) {
+  if (!out) {
+    set_error("out is NULL");
+    return EGGSYNC_EINVAL;
+  }
+  static const float dummy = 0.f;
+  EGG_TRY(validate(&dummy, n, d, eps));
+  EGG_TRY(check_device());
+  if (device >= 0) EGG_CUDA(cudaSetDevice(device));
+  eggsync_ctx* c = new eggsync_ctx();
+  int rc = c->ws.alloc(n, d, eps, device, (cudaStream_t)stream);
+  if (rc != EGGSYNC_OK) {
+    delete c;
+    return rc;
+  }
+  *out = c;
+  return EGGSYNC_OK;
+}
+
+void eggsync_ctx_destroy(eggsync_ctx* ctx) { delete ctx; }
+
+int eggsync_ctx_load(eggsync_ctx* ctx, const float* points, int32_t on_device) {
+  if (!ctx || !points) return EGGSYNC_EINVAL;
+  return stage_ingest(ctx->ws, points, on_device != 0);
+}
+
+int eggsync_ctx_build(eggsync_ctx* ctx, int32_t* n_cells_out) {
+  if (!ctx) return EGGSYNC_EINVAL;
+  Workspace& ws = ctx->ws;
+  EGG_TRY(stage_build(ws));
+  k_set_flags<<<1, 1, 0, ws.stream>>>(ws.flags, 1, 1);
+  EGG_CUDA(cudaGetLastError());
+  ws.second_checked = false;
+  if (n_cells_out) *n_cells_out = ws.n_cells;
+  return EGGSYNC_OK;
+}
+
+int eggsync_ctx_update(eggsync_ctx* ctx, int64_t lo, int64_t hi) {
+  if (!ctx || lo < 0 || hi > ctx->ws.n || lo > hi) return EGGSYNC_EINVAL;
+  if (!ctx->ws.built) {
+    set_error("eggsync_ctx_update before eggsync_ctx_build");
+    return EGGSYNC_EINVAL;
+  }
+  return stage_update(ctx->ws, lo, hi, nullptr);
+}
+
+int eggsync_ctx_second_term(eggsync_ctx* ctx, int64_t lo, int64_t hi) {
+  if (!ctx || lo < 0 || hi > ctx->ws.n || lo > hi) return EGGSYNC_EINVAL;
+  if (!ctx->ws.built) return EGGSYNC_EINVAL;
+  ctx->ws.second_checked = true;
+  return stage_second_term(ctx->ws, lo, hi);
+}
+
+int eggsync_ctx_flags(eggsync_ctx* ctx, int32_t* first_out, int32_t* second_out) {
+  if (!ctx) return EGGSYNC_EINVAL;
+  int32_t f1 = 0, f2 = 0;
+  EGG_TRY(read_flags(ctx->ws, &f1, &f2, nullptr));
+  if (first_out) *first_out = f1;
+  if (second_out) *second_out = ctx->ws.second_checked ? f2 : -1;
+  return EGGSYNC_OK;
+}
+
+float* eggsync_ctx_cur_coords(eggsync_ctx* ctx) { return ctx ? ctx->ws.xs[ctx->ws.xcur] : nullptr; }
+float* eggsync_ctx_next_coords(eggsync_ctx* ctx) { return ctx ? ctx->ws.xs[ctx->ws.xcur ^ 1] : nullptr; }
+
+int eggsync_ctx_pack(eggsync_ctx* ctx, int64_t lo, int64_t cnt, float* buf) {
+  if (!ctx || !buf || lo < 0 || cnt < 0) return EGGSYNC_EINVAL;
+  Workspace& ws = ctx->ws;
+  const int64_t tot = cnt * ws.d;
+  if (tot == 0) return EGGSYNC_OK;
+  k_pack<<<(unsigned)((tot + 255) / 256), 256, 0, ws.stream>>>(ws.xs[ws.xcur ^ 1], ws.n, ws.d, lo, cnt, buf);
+  EGG_CUDA(cudaGetLastError());
+  return EGGSYNC_OK;
+}
+
+int eggsync_ctx_unpack(eggsync_ctx* ctx, const float* gathered, int32_t ranks, int64_t cnt) {
+  if (!ctx || !gathered || ranks < 1 || cnt < 0) return EGGSYNC_EINVAL;
+  Workspace& ws = ctx->ws;
+  const int64_t tot = (int64_t)ranks * ws.d * cnt;
+  if (tot == 0) return EGGSYNC_OK;
+  k_unpack<<<(unsigned)((tot + 255) / 256), 256, 0, ws.stream>>>(gathered, ws.n, ws.d, ranks, cnt,
+                                                                  ws.xs[ws.xcur ^ 1]);
+  EGG_CUDA(cudaGetLastError());
+  return EGGSYNC_OK;
+}
+
+int eggsync_ctx_advance(eggsync_ctx* ctx) {
+  if (!ctx) return EGGSYNC_EINVAL;
+  advance(ctx->ws);
+  ctx->ws.have_final = false;
+  return EGGSYNC_OK;
+}
+
+int eggsync_ctx_labels(eggsync_ctx* ctx, int32_t* labels, int32_t on_device) {
+  if (!ctx || !labels) return EGGSYNC_EINVAL;
+  Workspace& ws = ctx->ws;
+  const int32_t* src = ws.lab_final;
+  if (!ws.have_final) {
+    if (!ws.built) EGG_TRY(stage_build(ws));
+    EGG_TRY(stage_labels(ws, ws.i_lab));
+    src = ws.i_lab;
+  }
+  EGG_CUDA(cudaMemcpyAsync(labels, src, sizeof(int32_t) * ws.n,
+                           on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, ws.stream));
+  EGG_CUDA(cudaStreamSynchronize(ws.stream));
+  return EGGSYNC_OK;
+}
+
+int eggsync_ctx_coords(eggsync_ctx* ctx, float* coords, int32_t on_device) {
+  if (!ctx || !coords) return EGGSYNC_EINVAL;
+  Workspace& ws = ctx->ws;
+  if (on_device) {
+    EGG_TRY(stage_coords(ws, ws.xcur, coords));
+  } else {
+    EGG_TRY(stage_coords(ws, ws.xcur, ws.io));
+    EGG_CUDA(cudaMemcpyAsync(coords, ws.io, sizeof(float) * ws.n * ws.d, cudaMemcpyDeviceToHost, ws.stream));
+  }
+  EGG_CUDA(cudaStreamSynchronize(ws.stream));
+  return EGGSYNC_OK;
+}
+
+int eggsync_ctx_run(eggsync_ctx* ctx, int32_t max_iters, int32_t* iters_out) {
+  if (!ctx || !iters_out || max_iters < 1) return EGGSYNC_EINVAL;
+  return run_loop(ctx->ws, max_iters, iters_out, nullptr);
+}
+
+void* eggsync_ctx_stream(eggsync_ctx* ctx) { return ctx ? (void*)ctx->ws.stream : nullptr; }
+
+}  // extern "C"

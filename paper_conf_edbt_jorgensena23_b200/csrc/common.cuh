@@ -1,0 +1,179 @@
+// common.cuh -- internal definitions of libeggsync (product path only).
+// Nothing here is shared with oracle/ (test infrastructure).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <cstdio>
+#include <string>
+
+#include "../../include/eggsync.h"
+
+namespace egg {
+
+constexpr int kMaxD = EGGSYNC_MAX_D;
+constexpr int kMaxKeyWords = 8;  // Morton keys up to 512 bits (d * ceil(log2 w))
+constexpr int kWarpsPerCta = 4;  // update / second-term CTAs: 4 independent warps
+constexpr int kBucket = 32;      // subtree of <= kBucket cells is processed cell by cell
+constexpr uint32_t kLeafBit = 0x80000000u;
+constexpr float kU = 5.9604644775390625e-08f;  // 2^-24, fp32 unit roundoff
+
+__host__ __device__ constexpr int ceil4(int x) { return (x + 3) & ~3; }
+
+// Hot-loop cell record in global memory (AoS, one per non-empty cell):
+//   [0, D)        centre of the cell's MBR (fp32)
+//   D             r = radius of the MBR about the centre (rounded up)
+//   D+1           count (int32 bits)
+//   D+2           start: first sorted position of the cell (int32 bits)
+//   [D+3, 2D+3)   sum_{q in cell} sin(q_i)  (fp32, rounded from the exact fixed-point sum)
+//   [2D+3, 3D+3)  sum_{q in cell} cos(q_i)
+template <int D>
+struct CellRec {
+  static constexpr int kFloats = ceil4(3 * D + 3);
+};
+
+// Per-warp staged cell layout in shared memory (floats):
+//   A: c'_0..c'_{D-1}, cc, lim_full, lim_out        (ceil4(D+3))
+//   B: ssin_0..ssin_{D-1}, scos_0..scos_{D-1}       (ceil4(2D))
+//   M: count, start (int bits), 2 pad               (4)
+template <int D>
+struct Stage {
+  static constexpr int kA = ceil4(D + 3);
+  static constexpr int kB = ceil4(2 * D);
+  static constexpr int kFloats = kA + kB + 4;
+};
+
+// Order-preserving map float -> uint32 (for deterministic atomic min/max of MBRs).
+__host__ __device__ inline uint32_t f2ord(float f) {
+  uint32_t b;
+  memcpy(&b, &f, 4);
+  return (b & 0x80000000u) ? ~b : (b | 0x80000000u);
+}
+__host__ __device__ inline float ord2f(uint32_t o) {
+  uint32_t b = (o & 0x80000000u) ? (o & 0x7fffffffu) : ~o;
+  float f;
+  memcpy(&f, &b, 4);
+  return f;
+}
+
+// Fixed-point scale for exact, order-independent cell / subtree sums of sin and cos
+// (values in [-1,1]; |sum| <= n * 2^32 < 2^63 for n < 2^31).
+constexpr double kFix = 4294967296.0;       // 2^32
+constexpr double kInvFix = 2.3283064365386963e-10;  // 2^-32
+
+// Run-time problem constants, all derived in fp64 from (double)eps.
+struct Consts {
+  int64_t n;
+  int d;
+  int bits;    // bits per dimension of a cell coordinate: ceil(log2 w), >= 1
+  int nw;      // 64-bit words per Morton key
+  int keybits; // d * bits
+  int64_t w;   // cells per dimension = ceil(1/c_w)          (Eq.4)
+  double e, e2, cw, inv_cw, delta, ed, ed2;  // eps, eps^2, c_w (L252), 1/c_w, delta (L110), eps+delta
+  float ef, e2f, edf, ed2f, rel;  // fp32 copies; rel = (4d+16) u relative safety margin
+};
+
+bool make_consts(int64_t n, int d, float eps, Consts* c, std::string* why);
+
+// thread-local error message
+void set_error(const char* fmt, ...);
+
+#define EGG_CUDA(call)                                                                   \
+  do {                                                                                   \
+    cudaError_t _e = (call);                                                             \
+    if (_e != cudaSuccess) {                                                             \
+      ::egg::set_error("%s failed: %s (%s:%d)", #call, cudaGetErrorString(_e), __FILE__, \
+                       __LINE__);                                                        \
+      return _e == cudaErrorMemoryAllocation ? EGGSYNC_ENOMEM : EGGSYNC_ECUDA;           \
+    }                                                                                    \
+  } while (0)
+
+#define EGG_TRY(expr)            \
+  do {                           \
+    int _rc = (expr);            \
+    if (_rc != EGGSYNC_OK) return _rc; \
+  } while (0)
+
+// ------------------------------------------------------------------ workspace
+struct Workspace {
+  Consts k;
+  int64_t n = 0;
+  int d = 0;
+  int64_t cap = 0;  // cell capacity (= n)
+  // state
+  float* xs[2] = {nullptr, nullptr};  // SoA [d][n] (sorted order)
+  uint32_t* orig[2] = {nullptr, nullptr};
+  int xcur = 0;  // xs[xcur] = D^t (sorted by its cell keys after build); xs[xcur^1] = D^{t+1}
+  int ocur = 0;  // orig[ocur] = original index of each sorted position of xs[xcur]
+  bool built = false;
+  // keys / sort
+  uint64_t* keys = nullptr;      // [nw][n] sorted
+  uint64_t* keys_tmp = nullptr;  // [nw][n]
+  uint64_t* kb[2] = {nullptr, nullptr};
+  uint32_t* pb[2] = {nullptr, nullptr};
+  void* cub_tmp = nullptr;
+  size_t cub_bytes = 0;
+  // per point
+  float* sn = nullptr;  // [d][n]
+  float* cs = nullptr;
+  int32_t* cell_of = nullptr;  // [n]
+  int32_t* iscan = nullptr;    // [n] int scratch
+  // cells
+  int32_t n_cells = 0;
+  int32_t* cell_start = nullptr;  // [cap+1]
+  uint64_t* c_fix = nullptr;      // [2d][cap]
+  uint32_t* c_lo = nullptr;       // [d][cap] ordered-float bits
+  uint32_t* c_hi = nullptr;
+  int32_t* c_cnt = nullptr;    // [cap]
+  float* c_rec = nullptr;      // [cap][CellRec<D>::kFloats]
+  uint64_t* c_key = nullptr;   // [nw][cap]
+  // tree (Karras radix tree over sorted cell keys; internal nodes 0..nc-2)
+  int4* t_meta = nullptr;      // first, last, left, right
+  int32_t* t_parent = nullptr; // [cap] parent of internal node
+  int32_t* l_parent = nullptr; // [cap] parent of leaf (cell)
+  uint32_t* t_visit = nullptr;
+  uint64_t* t_fix = nullptr;   // [2d][cap]
+  uint32_t* t_lo = nullptr;    // [d][cap]
+  uint32_t* t_hi = nullptr;
+  int32_t* t_cnt = nullptr;
+  float* t_box = nullptr;      // [cap][2d] lo then hi
+  float* t_sum = nullptr;      // [cap][2d] sin then cos
+  // flags: [0]=first term AND, [1]=second term AND, [2]=keys unsorted, [3]=error, [4]=domain error
+  int32_t* flags = nullptr;
+  int32_t* h_flags = nullptr;  // pinned host mirror
+  // io scratch
+  float* io = nullptr;         // n*d row-major staging (device)
+  int32_t* i_lab = nullptr;    // [n] labels scratch
+  uint32_t* c_minorig = nullptr;
+  int32_t* nbr = nullptr;      // optional neighbour counts (sorted order)
+  int32_t* lab_final = nullptr; // labels recorded when the criterion held (original order)
+  bool have_final = false;
+  bool second_checked = false;
+  int64_t bytes = 0;
+  char* arena = nullptr;  // one device allocation carved into the arrays above
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  int device = 0;
+  cudaEvent_t ev[8];
+  bool ev_ok = false;
+  int sort_skipped = 0;
+
+  int alloc(int64_t n, int d, float eps, int device, cudaStream_t stream);
+  void release();
+  ~Workspace() { release(); }
+};
+
+// ------------------------------------------------------------ pipeline stages
+int stage_ingest(Workspace& ws, const float* points, bool on_device);
+int stage_build(Workspace& ws);  // keys, sort, segment, summaries, tree
+int stage_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr_sorted);
+int stage_second_term(Workspace& ws, int64_t lo, int64_t hi);
+int stage_labels(Workspace& ws, int32_t* labels_dev);  // labels of current cells, original order
+int stage_coords(Workspace& ws, int which, float* out_dev);  // row-major, original order
+int stage_scatter_i32(Workspace& ws, const int32_t* sorted_vals, int32_t* out_dev);
+
+// dispatch helpers (templated on D in update.cu / term.cu / grid.cu)
+int launch_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr_sorted);
+int launch_second_term(Workspace& ws, int64_t lo, int64_t hi);
+
+}  // namespace egg

@@ -1,0 +1,183 @@
+// term.cuh -- A7b: second term of the synchronization criterion (Def 4.2,
+// PAPER.md L106-110; its grid check L254), evaluated only when the first term
+// holds (Alg 4 l.9-10, L273-275).
+//
+// Violation iff for some p there is q with eps < ||p-q|| <= eps + delta and
+// dist(MBR(N_{eps/2}(q)), p) <= eps.  When the first term holds in its grid
+// form every neighbourhood is exactly a cell (diagonal <= eps/2, L252), so
+// N_{eps/2}(q) = cell(q) and its MBR is the cell MBR computed in A4.  The
+// search uses the same subtree hierarchy as the update with radius eps+delta.
+#pragma once
+#include "update.cuh"
+
+namespace egg {
+
+template <int D>
+struct TermArgs {
+  const float* __restrict__ xs;
+  const int32_t* __restrict__ cell_of;
+  const int32_t* __restrict__ cell_start;
+  const uint32_t* __restrict__ c_lo;
+  const uint32_t* __restrict__ c_hi;
+  const int4* __restrict__ t_meta;
+  const float* __restrict__ t_box;
+  int64_t n, cap, lo, hi;
+  int32_t nc, stack_len;
+  float e2f, ed2f, rel;
+  double e2d, ed2d;
+  int32_t* flags;  // [1] second term AND, [3] error
+};
+
+// dist(MBR, p)^2 exactly as the oracle evaluates it (L110; fp64, dimension order)
+template <int D>
+__device__ __forceinline__ double exact_mindist2(const float* lo, const float* hi, const float* p) {
+  double m = 0.0;
+#pragma unroll
+  for (int i = 0; i < D; ++i) {
+    const double v = (double)p[i], l = (double)lo[i], h = (double)hi[i];
+    double t = 0.0;
+    if (v < l) t = __dsub_rn(l, v);
+    else if (v > h) t = __dsub_rn(v, h);
+    m = __dadd_rn(m, __dmul_rn(t, t));
+  }
+  return m;
+}
+
+template <int D>
+__global__ void __launch_bounds__(kWarpsPerCta * 32) k_second(const TermArgs<D> a) {
+  constexpr int BS = ceil4(2 * D);
+  extern __shared__ __align__(16) float smem[];
+  const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  int2* stk = reinterpret_cast<int2*>(smem) + wid * a.stack_len;
+  const int64_t j = a.lo + ((int64_t)blockIdx.x * kWarpsPerCta + wid) * 32 + lane;
+  const bool valid = j < a.hi;
+  const unsigned amask = __ballot_sync(FULLMASK, valid);
+  if (amask == 0u) return;
+  float p[D];
+#pragma unroll
+  for (int i = 0; i < D; ++i) p[i] = valid ? a.xs[(int64_t)i * a.n + j] : 0.f;
+  const int32_t own = valid ? a.cell_of[j] : -1;
+  const float lim_ed = a.ed2f * (1.f + a.rel);
+  const float e_in = a.e2f * (1.f - a.rel), e_out = a.e2f * (1.f + a.rel);
+  const float ed_in = a.ed2f * (1.f - a.rel);
+  bool viol = false;
+  int sp = 1;
+  if (lane == 0) stk[0] = make_int2(a.nc > 1 ? 0 : (int)kLeafBit, (int)amask);
+  __syncwarp();
+  while (sp > 0) {
+    if (*(volatile int32_t*)&a.flags[1] == 0) break;  // someone already found a violation
+    --sp;
+    const int2 ent = stk[sp];
+    __syncwarp();
+    const unsigned m = (unsigned)ent.y;
+    const bool act = (m >> lane) & 1u;
+    int32_t first, last;
+    unsigned pm;
+    if (ent.x & (int)kLeafBit) {
+      first = last = ent.x & 0x7fffffff;
+      pm = m;
+    } else {
+      const float* __restrict__ bx = a.t_box + (int64_t)ent.x * BS;
+      float mind = 0.f;
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        const float mn = fmaxf(fmaxf(bx[i] - p[i], p[i] - bx[D + i]), 0.f);
+        mind = fmaf(mn, mn, mind);
+      }
+      pm = __ballot_sync(FULLMASK, act && mind <= lim_ed);
+      if (pm == 0u) continue;
+      const int4 meta = a.t_meta[ent.x];
+      if (meta.y - meta.x + 1 > kBucket) {
+        if (sp + 2 > a.stack_len) {
+          if (lane == 0) atomicExch(&a.flags[3], 1);
+          break;
+        }
+        if (lane == 0) {
+          stk[sp] = make_int2(meta.w, (int)pm);
+          stk[sp + 1] = make_int2(meta.z, (int)pm);
+        }
+        sp += 2;
+        __syncwarp();
+        continue;
+      }
+      first = meta.x;
+      last = meta.y;
+    }
+    const bool pact = (pm >> lane) & 1u;
+    for (int32_t c = first; c <= last; ++c) {
+      float lo[D], hi[D];
+      float mind = 0.f;
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        lo[i] = ordf(a.c_lo[(int64_t)i * a.cap + c]);
+        hi[i] = ordf(a.c_hi[(int64_t)i * a.cap + c]);
+        const float mn = fmaxf(fmaxf(lo[i] - p[i], p[i] - hi[i]), 0.f);
+        mind = fmaf(mn, mn, mind);
+      }
+      // condition on q's MBR: dist(MBR(cell(q)), p) <= eps (L108), decided exactly near the margin
+      bool cand = pact && c != own && mind <= e_out;
+      const bool amb = cand && mind > e_in;
+      if (__any_sync(FULLMASK, amb)) {
+        if (amb) cand = exact_mindist2<D>(lo, hi, p) <= a.e2d;
+      }
+      if (!__any_sync(FULLMASK, cand)) continue;
+      const int32_t s0 = a.cell_start[c], s1 = a.cell_start[c + 1];
+      for (int32_t q = s0; q < s1; ++q) {
+        float qv[D];
+        float d2 = 0.f;
+#pragma unroll
+        for (int i = 0; i < D; ++i) {
+          qv[i] = a.xs[(int64_t)i * a.n + q];
+          const float t = qv[i] - p[i];
+          d2 = fmaf(t, t, d2);
+        }
+        // eps < ||p-q|| <= eps + delta   (L108)
+        bool shell = cand && d2 > e_out && d2 <= ed_in;
+        const bool amb2 = cand && !shell && d2 > e_in && d2 <= lim_ed;
+        if (__any_sync(FULLMASK, amb2)) {
+          if (amb2) {
+            const double x = exact_d2<D>(qv, p);
+            shell = x > a.e2d && x <= a.ed2d;
+          }
+        }
+        viol = viol || shell;
+      }
+      if (__any_sync(FULLMASK, viol)) break;
+    }
+    if (__any_sync(FULLMASK, viol)) break;
+  }
+  if (__any_sync(FULLMASK, viol) && lane == 0) atomicAnd(&a.flags[1], 0);
+}
+
+template <int D>
+int run_second_term(Workspace& ws, int64_t lo, int64_t hi) {
+  if (hi <= lo) return EGGSYNC_OK;
+  TermArgs<D> a;
+  a.xs = ws.xs[ws.xcur];
+  a.cell_of = ws.cell_of;
+  a.cell_start = ws.cell_start;
+  a.c_lo = ws.c_lo;
+  a.c_hi = ws.c_hi;
+  a.t_meta = ws.t_meta;
+  a.t_box = ws.t_box;
+  a.n = ws.n;
+  a.cap = ws.cap;
+  a.lo = lo;
+  a.hi = hi;
+  a.nc = ws.n_cells;
+  a.stack_len = ws.k.keybits + 4;
+  a.e2f = ws.k.e2f;
+  a.ed2f = ws.k.ed2f;
+  a.rel = ws.k.rel;
+  a.e2d = ws.k.e2;
+  a.ed2d = ws.k.ed2;
+  a.flags = ws.flags;
+  const size_t smem = (size_t)kWarpsPerCta * a.stack_len * sizeof(int2);
+  EGG_CUDA(cudaFuncSetAttribute(k_second<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  const int64_t per = 32 * kWarpsPerCta;
+  k_second<D><<<(unsigned)((hi - lo + per - 1) / per), kWarpsPerCta * 32, smem, ws.stream>>>(a);
+  EGG_CUDA(cudaGetLastError());
+  return EGGSYNC_OK;
+}
+
+}  // namespace egg

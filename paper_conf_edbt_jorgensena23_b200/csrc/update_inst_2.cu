@@ -1,0 +1,21 @@
+// update_inst_2.cu -- explicit instantiations of the update and second-term kernels, D=17..24.
+// (split across files so the 32 dimension variants compile in parallel)
+#include "term.cuh"
+namespace egg {
+template int run_update<17>(Workspace&, int64_t, int64_t, int32_t*);
+template int run_second_term<17>(Workspace&, int64_t, int64_t);
+template int run_update<18>(Workspace&, int64_t, int64_t, int32_t*);
+template int run_second_term<18>(Workspace&, int64_t, int64_t);
+template int run_update<19>(Workspace&, int64_t, int64_t, int32_t*);
+template int run_second_term<19>(Workspace&, int64_t, int64_t);
+template int run_update<20>(Workspace&, int64_t, int64_t, int32_t*);
+template int run_second_term<20>(Workspace&, int64_t, int64_t);
+template int run_update<21>(Workspace&, int64_t, int64_t, int32_t*);
+template int run_second_term<21>(Workspace&, int64_t, int64_t);
+template int run_update<22>(Workspace&, int64_t, int64_t, int32_t*);
+template int run_second_term<22>(Workspace&, int64_t, int64_t);
+template int run_update<23>(Workspace&, int64_t, int64_t, int32_t*);
+template int run_second_term<23>(Workspace&, int64_t, int64_t);
+template int run_update<24>(Workspace&, int64_t, int64_t, int32_t*);
+template int run_second_term<24>(Workspace&, int64_t, int64_t);
+}  // namespace egg

@@ -1,0 +1,271 @@
+"""Thin ctypes binding of libeggsync.so (include/eggsync.h).
+
+Argument marshalling only: every step of the method runs in the library's
+CUDA kernels.  Host inputs are numpy arrays; device inputs are CUDA torch
+tensors (their data pointers are passed with ``device_pointers=1``).  There
+is no CPU fallback -- if the library or a CUDA device is missing, calls raise.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libeggsync.so")
+
+OK, NOT_CONVERGED, EINVAL, EDOMAIN, ENOMEM, ECUDA, ENCCL = 0, 1, -1, -2, -3, -4, -5
+MAX_D = 32
+
+#: every symbol include/eggsync.h declares
+SYMBOLS = [
+    "eggsync_default_opts", "eggsync_cluster", "eggsync_cluster_ex", "eggsync_step", "eggsync_step_ex",
+    "eggsync_last_error", "eggsync_version", "eggsync_ctx_create", "eggsync_ctx_destroy",
+    "eggsync_ctx_load", "eggsync_ctx_build", "eggsync_ctx_update", "eggsync_ctx_second_term",
+    "eggsync_ctx_flags", "eggsync_ctx_cur_coords", "eggsync_ctx_next_coords", "eggsync_ctx_pack",
+    "eggsync_ctx_unpack", "eggsync_ctx_advance", "eggsync_ctx_labels", "eggsync_ctx_coords",
+    "eggsync_ctx_run", "eggsync_ctx_stream",
+]
+
+
+class EggSyncError(RuntimeError):
+    def __init__(self, rc: int, msg: str):
+        super().__init__(f"eggsync error {rc}: {msg}")
+        self.rc = rc
+
+
+class Stats(ctypes.Structure):
+    """eggsync_stats: Table 1 columns (L364-371) + counters."""
+    _fields_ = [("t_alloc", ctypes.c_double), ("t_build", ctypes.c_double), ("t_update", ctypes.c_double),
+                ("t_extra_check", ctypes.c_double), ("t_cluster", ctypes.c_double),
+                ("t_free", ctypes.c_double), ("t_transfer", ctypes.c_double), ("iters", ctypes.c_int32),
+                ("n_cells_first", ctypes.c_int32), ("n_cells_last", ctypes.c_int32),
+                ("sort_skipped", ctypes.c_int32), ("device_bytes", ctypes.c_int64)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class Opts(ctypes.Structure):
+    _fields_ = [("struct_size", ctypes.c_int32), ("max_iters", ctypes.c_int32), ("device", ctypes.c_int32),
+                ("device_pointers", ctypes.c_int32), ("stream", ctypes.c_void_p), ("term_mode", ctypes.c_int32),
+                ("coords_out", ctypes.c_void_p), ("nbr_count_out", ctypes.c_void_p),
+                ("stats", ctypes.POINTER(Stats))]
+
+
+_lib = None
+
+
+def lib():
+    """Load the CUDA library; fail loudly if it has not been built (no fallback)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} missing: run `python -c 'import __graft_entry__ as g; g.build()'`")
+        L = ctypes.CDLL(LIB_PATH)
+        vp, i64, i32, f32 = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int32, ctypes.c_float
+        sig = {
+            "eggsync_default_opts": ([vp], None),
+            "eggsync_cluster": ([vp, i64, i32, f32, vp, vp], ctypes.c_int),
+            "eggsync_cluster_ex": ([vp, i64, i32, f32, vp, vp, vp], ctypes.c_int),
+            "eggsync_step": ([vp, i64, i32, f32, vp], ctypes.c_int),
+            "eggsync_step_ex": ([vp, i64, i32, f32, vp, vp, vp], ctypes.c_int),
+            "eggsync_last_error": ([], ctypes.c_char_p),
+            "eggsync_version": ([], ctypes.c_char_p),
+            "eggsync_ctx_create": ([i64, i32, f32, i32, vp, ctypes.POINTER(vp)], ctypes.c_int),
+            "eggsync_ctx_destroy": ([vp], None),
+            "eggsync_ctx_load": ([vp, vp, i32], ctypes.c_int),
+            "eggsync_ctx_build": ([vp, vp], ctypes.c_int),
+            "eggsync_ctx_update": ([vp, i64, i64], ctypes.c_int),
+            "eggsync_ctx_second_term": ([vp, i64, i64], ctypes.c_int),
+            "eggsync_ctx_flags": ([vp, vp, vp], ctypes.c_int),
+            "eggsync_ctx_cur_coords": ([vp], vp),
+            "eggsync_ctx_next_coords": ([vp], vp),
+            "eggsync_ctx_pack": ([vp, i64, i64, vp], ctypes.c_int),
+            "eggsync_ctx_unpack": ([vp, vp, i32, i64], ctypes.c_int),
+            "eggsync_ctx_advance": ([vp], ctypes.c_int),
+            "eggsync_ctx_labels": ([vp, vp, i32], ctypes.c_int),
+            "eggsync_ctx_coords": ([vp, vp, i32], ctypes.c_int),
+            "eggsync_ctx_run": ([vp, i32, vp], ctypes.c_int),
+            "eggsync_ctx_stream": ([vp], vp),
+        }
+        for name, (args, res) in sig.items():
+            fn = getattr(L, name)
+            fn.argtypes = args
+            fn.restype = res
+        _lib = L
+    return _lib
+
+
+def last_error() -> str:
+    return lib().eggsync_last_error().decode()
+
+
+def _check(rc: int, allow=(OK,)):
+    if rc not in allow:
+        raise EggSyncError(rc, last_error())
+    return rc
+
+
+def _is_torch_cuda(x):
+    return type(x).__module__.startswith("torch") and getattr(x, "is_cuda", False)
+
+
+def _ptr(a):
+    if _is_torch_cuda(a):
+        return ctypes.c_void_p(a.data_ptr())
+    return a.ctypes.data_as(ctypes.c_void_p)
+
+
+def default_opts() -> Opts:
+    o = Opts()
+    lib().eggsync_default_opts(ctypes.byref(o))
+    return o
+
+
+def _host_points(points, writable=False):
+    a = np.ascontiguousarray(points, dtype=np.float32)
+    if a.ndim != 2:
+        raise ValueError("points must be (n, d)")
+    if writable and a is points:
+        return a
+    return a.copy() if writable else a
+
+
+def cluster(points, eps: float, *, max_iters: int = 10000, coords: bool = False, stats: bool = False,
+            stream=None):
+    """EGG-SynC clustering (Alg 4).  points: (n,d) float32 numpy (host) or CUDA torch tensor.
+
+    Returns dict(labels, iters, converged[, coords][, stats]).  Device inputs give device outputs.
+    """
+    dev = _is_torch_cuda(points)
+    o = default_opts()
+    o.max_iters = max_iters
+    if dev:
+        import torch
+        assert points.dtype == torch.float32 and points.is_contiguous() and points.dim() == 2
+        n, d = points.shape
+        o.device_pointers = 1
+        o.device = points.device.index
+        o.stream = ctypes.c_void_p(stream if stream is not None else torch.cuda.current_stream(points.device).cuda_stream)
+        labels = torch.empty(n, dtype=torch.int32, device=points.device)
+        co = torch.empty((n, d), dtype=torch.float32, device=points.device) if coords else None
+    else:
+        points = _host_points(points)
+        n, d = points.shape
+        labels = np.empty(n, np.int32)
+        co = np.empty((n, d), np.float32) if coords else None
+    st = Stats()
+    if stats:
+        o.stats = ctypes.pointer(st)
+    if co is not None:
+        o.coords_out = _ptr(co)
+    iters = ctypes.c_int32(0)
+    rc = lib().eggsync_cluster_ex(_ptr(points), n, d, ctypes.c_float(eps), ctypes.byref(o), _ptr(labels),
+                                  ctypes.byref(iters))
+    _check(rc, (OK, NOT_CONVERGED))
+    out = {"labels": labels, "iters": iters.value, "converged": rc == OK}
+    if coords:
+        out["coords"] = co
+    if stats:
+        out["stats"] = st.as_dict()
+    return out
+
+
+def step(points, eps: float, *, nbr: bool = False):
+    """One Eq.1 update (eggsync_step_ex) of host points.  Returns dict(points, first, second, synced[, nbr])."""
+    x = _host_points(points, writable=True)
+    n, d = x.shape
+    o = default_opts()
+    cnt = np.empty(n, np.int32) if nbr else None
+    if nbr:
+        o.nbr_count_out = _ptr(cnt)
+    f1, f2 = ctypes.c_int32(0), ctypes.c_int32(0)
+    _check(lib().eggsync_step_ex(_ptr(x), n, d, ctypes.c_float(eps), ctypes.byref(o), ctypes.byref(f1),
+                                 ctypes.byref(f2)))
+    out = {"points": x, "first": f1.value, "second": f2.value, "synced": int(f1.value == 1 and f2.value == 1)}
+    if nbr:
+        out["nbr"] = cnt
+    return out
+
+
+class Context:
+    """Device-resident phase API (eggsync_ctx_*), used by the multi-GPU driver and device-timed bench."""
+
+    def __init__(self, n: int, d: int, eps: float, device: int = -1, stream=None):
+        self.n, self.d, self.eps = n, d, eps
+        h = ctypes.c_void_p()
+        _check(lib().eggsync_ctx_create(n, d, ctypes.c_float(eps), device,
+                                        ctypes.c_void_p(stream) if stream else None, ctypes.byref(h)))
+        self.h = h
+
+    def close(self):
+        if self.h:
+            lib().eggsync_ctx_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def load(self, points):
+        on_dev = _is_torch_cuda(points)
+        if not on_dev:
+            points = _host_points(points)
+        self._keep = points
+        _check(lib().eggsync_ctx_load(self.h, _ptr(points), int(on_dev)))
+
+    def build(self) -> int:
+        nc = ctypes.c_int32(0)
+        _check(lib().eggsync_ctx_build(self.h, ctypes.byref(nc)))
+        return nc.value
+
+    def update(self, lo: int = 0, hi: int | None = None):
+        _check(lib().eggsync_ctx_update(self.h, lo, self.n if hi is None else hi))
+
+    def second_term(self, lo: int = 0, hi: int | None = None):
+        _check(lib().eggsync_ctx_second_term(self.h, lo, self.n if hi is None else hi))
+
+    def flags(self):
+        a, b = ctypes.c_int32(0), ctypes.c_int32(0)
+        _check(lib().eggsync_ctx_flags(self.h, ctypes.byref(a), ctypes.byref(b)))
+        return a.value, b.value
+
+    def next_coords_ptr(self) -> int:
+        return lib().eggsync_ctx_next_coords(self.h)
+
+    def cur_coords_ptr(self) -> int:
+        return lib().eggsync_ctx_cur_coords(self.h)
+
+    def pack(self, lo: int, cnt: int, buf_ptr: int):
+        _check(lib().eggsync_ctx_pack(self.h, lo, cnt, ctypes.c_void_p(buf_ptr)))
+
+    def unpack(self, gathered_ptr: int, ranks: int, cnt: int):
+        _check(lib().eggsync_ctx_unpack(self.h, ctypes.c_void_p(gathered_ptr), ranks, cnt))
+
+    def advance(self):
+        _check(lib().eggsync_ctx_advance(self.h))
+
+    def labels(self, out=None):
+        if out is None:
+            out = np.empty(self.n, np.int32)
+        _check(lib().eggsync_ctx_labels(self.h, _ptr(out), int(_is_torch_cuda(out))))
+        return out
+
+    def coords(self, out=None):
+        if out is None:
+            out = np.empty((self.n, self.d), np.float32)
+        _check(lib().eggsync_ctx_coords(self.h, _ptr(out), int(_is_torch_cuda(out))))
+        return out
+
+    def run(self, max_iters: int = 10000):
+        it = ctypes.c_int32(0)
+        rc = lib().eggsync_ctx_run(self.h, max_iters, ctypes.byref(it))
+        _check(rc, (OK, NOT_CONVERGED))
+        return it.value, rc == OK
+
+    def stream(self) -> int:
+        return lib().eggsync_ctx_stream(self.h) or 0

@@ -1,0 +1,86 @@
+"""C-ABI boundary tests that need no GPU: the library loads, exports every
+symbol include/eggsync.h declares, and argument validation returns the
+documented codes before touching any device or output buffer."""
+import ctypes
+import os
+import re
+
+import numpy as np
+import pytest
+
+from paper_conf_edbt_jorgensena23_b200 import eggsync as E
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "eggsync.h")
+
+
+def _declared():
+    src = open(HEADER).read()
+    src = re.sub(r"/\*.*?\*/", "", src, flags=re.S)
+    return sorted(set(re.findall(r"\b(eggsync_[a-z_]+)\s*\(", src)))
+
+
+def test_library_exports_every_declared_symbol():
+    L = E.lib()
+    names = _declared()
+    assert len(names) >= 20
+    for nm in names:
+        assert hasattr(L, nm), nm
+    assert sorted(E.SYMBOLS) == names
+
+
+def test_library_is_sm100a_and_has_no_host_fallback():
+    out = os.popen(f"/usr/local/cuda/bin/cuobjdump --list-elf {E.LIB_PATH} 2>&1").read()
+    assert "sm_100a" in out
+    assert E.lib().eggsync_version().decode().endswith("(sm_100a)")
+
+
+def test_default_opts():
+    o = E.default_opts()
+    assert o.struct_size == ctypes.sizeof(E.Opts)
+    assert o.max_iters == 10000 and o.device == -1 and o.device_pointers == 0
+
+
+@pytest.mark.parametrize("n,d,eps", [(0, 2, 0.05), (10, 0, 0.05), (10, 33, 0.05), (10, 2, 0.0),
+                                     (10, 2, float("nan")), (10, 2, float("inf")), (10, 2, -1.0),
+                                     (2 ** 31, 2, 0.05), (10, 32, 1e-7)])
+def test_invalid_arguments_return_einval_and_leave_outputs(n, d, eps):
+    pts = np.full((2, 2), 0.5, np.float32)
+    lab = np.full(2, -7, np.int32)
+    it = ctypes.c_int32(-9)
+    rc = E.lib().eggsync_cluster(pts.ctypes.data_as(ctypes.c_void_p), n, d, ctypes.c_float(eps),
+                                 lab.ctypes.data_as(ctypes.c_void_p), ctypes.byref(it))
+    assert rc == E.EINVAL, E.last_error()
+    assert (lab == -7).all() and it.value == -9
+    assert E.last_error()
+
+
+def test_null_pointers_are_einval():
+    L = E.lib()
+    it = ctypes.c_int32(0)
+    assert L.eggsync_cluster(None, 10, 2, ctypes.c_float(0.05), None, ctypes.byref(it)) == E.EINVAL
+    lab = np.zeros(10, np.int32)
+    pts = np.zeros((10, 2), np.float32)
+    assert L.eggsync_cluster(pts.ctypes.data_as(ctypes.c_void_p), 10, 2, ctypes.c_float(0.05), None,
+                             ctypes.byref(it)) == E.EINVAL
+    assert L.eggsync_step(None, 10, 2, ctypes.c_float(0.05), None) == E.EINVAL
+
+
+def test_bad_opts_struct_size():
+    o = E.default_opts()
+    o.struct_size = 3
+    pts = np.zeros((4, 2), np.float32)
+    lab = np.zeros(4, np.int32)
+    it = ctypes.c_int32(0)
+    rc = E.lib().eggsync_cluster_ex(pts.ctypes.data_as(ctypes.c_void_p), 4, 2, ctypes.c_float(0.05),
+                                    ctypes.byref(o), lab.ctypes.data_as(ctypes.c_void_p), ctypes.byref(it))
+    assert rc == E.EINVAL
+
+
+def test_no_cpu_fallback_without_device(cuda_available):
+    if cuda_available:
+        pytest.skip("device present")
+    with pytest.raises(E.EggSyncError) as ei:
+        E.cluster(np.full((8, 2), 0.5, np.float32), 0.05)
+    assert ei.value.rc == E.ECUDA
+    assert "no CUDA device" in str(ei.value)
