@@ -128,9 +128,7 @@ def _host_points(points, writable=False):
     a = np.ascontiguousarray(points, dtype=np.float32)
     if a.ndim != 2:
         raise ValueError("points must be (n, d)")
-    if writable and a is points:
-        return a
-    return a.copy() if writable else a
+    return a.copy() if writable else a  # step() writes D^{t+1}: never alias the caller's array
 
 
 def cluster(points, eps: float, *, max_iters: int = 10000, coords: bool = False, stats: bool = False,

@@ -74,7 +74,8 @@ def test_step_boundary_pairs():
     X = np.array([[0.0, 0.5], [e, 0.5], [0.3, 0.3], [0.3 + np.nextafter(e, np.float32(1)), 0.3],
                   [1.0, 1.0], [1.0 - e, 1.0]], np.float32)
     g = _step_compare(X, float(e))
-    assert g["nbr"].tolist() == [2, 2, 1, 1, 2, 2]
+    # 1.0 - fl32(1 - e) = 0.0500000119 > e: the last pair is NOT within eps (fp32 input rounding)
+    assert g["nbr"].tolist() == [2, 2, 1, 1, 1, 1]
 
 
 @pytest.mark.parametrize("name", [k for k in GOLD if not k.startswith("_")])
