@@ -1,0 +1,334 @@
+#!/usr/bin/env python
+"""Benchmark of the EGG-SynC synchronization update on B200 (BASELINE.json metric).
+
+One step = one complete EGG-SynC clustering (all §8(a) rows: keys, sort, cell
+offsets, summaries, hierarchy, update, both criterion terms, labels) of the
+workload BASELINE.json's metric is quoted on: C3, n=1,000,000, d=10, 20
+Gaussian clusters + 5% uniform noise, eps=0.1 (synthetic, seed 0).
+
+  value  = point-updates/s = n * iters / device time of the step (inputs
+           resident in HBM; L2 flushed by a 256 MiB write between steps)
+  e2e    = the same metric through eggsync_cluster() with pinned HOST
+           buffers (H2D of the points and D2H of the labels inside the timing)
+
+Usage:  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+        (N>1: launched under torch.distributed.run, one rank per GPU, NCCL)
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+METRIC = "end-to-end clustering sec and point-updates/sec at n=1M,d=10; 1/2/4/8 B200"
+UNIT = "point-updates/s"
+PEAKS_PATH = os.path.join(ROOT, "MEASURED_PEAKS.json")
+SM_COUNT, FP32_LANES = 148, 128
+
+
+def workload_desc(c):
+    return (f"{c.name}: n={c.n:,} d={c.d} {c.k} Gaussian clusters (std 5 in [-100,100]^d)"
+            f" + {int(c.noise * 100)}% uniform noise, min/max-normalised, eps={c.eps}, seed 0")
+
+
+# ----------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks and throttle reasons during the timed region (B200_PROFILING.md)."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index, self.rows, self.proc = index, [], None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-i", str(self.index), "-lms", "200"], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except FileNotFoundError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 7:
+                self.rows.append(parts)
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[k] for r in self.rows for k in range(4) if r[3 + k].lower() == "active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+# -------------------------------------------------------- cpu baseline
+def oracle_rate(X, eps, target_s: float, seed: int = 0):
+    """The fp64 oracle (as it stands) on a bounded sample: Eq.1 updates of m sampled points
+    against the full state (oracle_step_sample).  Returns (point-updates/s, m, seconds, cores)."""
+    import oracle
+    rng = np.random.default_rng(seed)
+    m = 8
+    while True:
+        idx = rng.choice(len(X), m, replace=False)
+        t0 = time.perf_counter()
+        oracle.step_sample(X, eps, idx)
+        dt = time.perf_counter() - t0
+        if dt >= 0.25 * target_s or m >= len(X):
+            return m / dt, m, dt, os.cpu_count()
+        m = int(min(len(X), max(m * 2, m * 0.3 * target_s / max(dt, 1e-3))))
+
+
+def cpu_baseline_obj(X, c, target_s):
+    rate, m, dt, cores = oracle_rate(X, c.eps, target_s)
+    return {"value": rate, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{m} Eq.1 point-updates of {c.name} iteration 1 (each against the full n={c.n:,} state), "
+                      f"fp64 C/OpenMP oracle, {dt:.1f} s on {cores} threads"}
+
+
+# ------------------------------------------------------------- helpers
+def dist_env():
+    return int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0")), \
+        int(os.environ.get("LOCAL_RANK", "0"))
+
+
+def load_peaks():
+    try:
+        return json.load(open(PEAKS_PATH))
+    except Exception:
+        return None
+
+
+def work_flops(w, d):
+    """Algorithmic FP32 FLOPs of the update: squared distance to a staged
+    cell 2d (d FMA), accumulation of a summary / neighbour 2d (adds), scanned-point distance 3d,
+    subtree box test (min+max distance) 6d."""
+    return 2 * d * w["cls"] + 2 * d * w["acc"] + 3 * d * w["scan"] + 6 * d * w["node"]
+
+
+def traffic_from_profiles():
+    p = os.path.join(ROOT, "profiles", "ncu_update_traffic.json")
+    try:
+        return json.load(open(p)).get("bytes_per_launch")
+    except Exception:
+        return None
+
+
+# ------------------------------------------------------------ our arm
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_edbt_jorgensena23_b200 import datagen, distributed as DR, eggsync as E
+
+    world, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    c = datagen.make_config(args.config)
+    X = c.generate(args.seed)
+    n, d = X.shape
+    stream = torch.cuda.current_stream(dev)
+    Xd = torch.from_numpy(X).to(dev)
+    ctx = E.Context(n, d, c.eps, device=local, stream=stream.cuda_stream)
+    comm = DR.TorchComm(n, d, dev) if world > 1 else DR.LocalComm(n)
+    flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
+
+    class Hooks:
+        def __init__(self):
+            self.ev = []
+
+        def before_update(self):
+            e = torch.cuda.Event(enable_timing=True)
+            e.record(stream)
+            self.ev.append([e, None])
+
+        def after_update(self):
+            e = torch.cuda.Event(enable_timing=True)
+            e.record(stream)
+            self.ev[-1][1] = e
+
+    def one_step(hooks=None):
+        ctx.load(Xd)
+        it, ok, lab = DR.run(ctx, comm, hooks=hooks)
+        return it, ok, lab
+
+    for _ in range(args.warmup):
+        flush.zero_()
+        it, ok, lab = one_step()
+    assert ok, "clustering did not converge"
+    # instrumented pass (untimed): algorithmic work of the update launches
+    ctx.work(enable=1)
+    one_step()
+    work = ctx.work(enable=0)
+    # timed region
+    hooks = Hooks()
+    step_ms = []
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    launches0 = ctx.launches()
+    with ClockSampler(local) as clk:
+        for _ in range(args.steps):
+            flush.zero_()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            it, ok, lab = one_step(hooks)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            step_ms.append(e0.elapsed_time(e1))
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    launches = ctx.launches() - launches0
+    upd_ms = [a.elapsed_time(b) for a, b in hooks.ev]
+    ms = statistics.mean(step_ms)
+    if world > 1:
+        t = torch.tensor([ms, sum(upd_ms) / len(upd_ms)], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms, upd_avg = float(t[0]), float(t[1])
+    else:
+        upd_avg = sum(upd_ms) / len(upd_ms)
+    iters = it
+    value = n * iters / (ms / 1e3)
+
+    # roofline of the dominant kernel (k_update): FP32 pipe
+    flops_per_launch = work_flops(work, d) / iters  # per launch on this rank (its range share)
+    achieved = flops_per_launch / (upd_avg / 1e3) / 1e12
+    peaks = load_peaks()
+    clk_s = clk.summary()
+    fmax = (peaks or {}).get("sm_max_mhz") or clk_s["sm_max_mhz"] or 1965.0
+    peak = 2 * FP32_LANES * SM_COUNT * fmax * 1e6 / 1e12
+    upd_share = sum(upd_ms) / sum(step_ms)
+
+    # end-to-end through the C ABI with pinned host buffers (rank 0 at N=1 only)
+    e2e = None
+    cpu = None
+    if world == 1 and not args.no_e2e:
+        pin = torch.empty((n, d), dtype=torch.float32, pin_memory=True)
+        pin.numpy()[:] = X
+        Xp = pin.numpy()
+        lab_pin = torch.empty(n, dtype=torch.int32, pin_memory=True).numpy()
+        ts = []
+        for k in range(args.warmup + args.steps):
+            flush.zero_()
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            r = E.cluster(Xp, c.eps)
+            dt = time.perf_counter() - t0
+            lab_pin[:] = r["labels"]
+            if k >= args.warmup:
+                ts.append(dt)
+        te = statistics.mean(ts)
+        e2e = {"value": n * r["iters"] / te, "unit": UNIT, "h2d_bytes_per_step": int(n * d * 4),
+               "d2h_bytes_per_step": int(n * 4), "seconds": te,
+               "how": "wall time of the synchronous eggsync_cluster() call from pinned host points to host labels "
+                      "(workspace alloc/free, H2D, all iterations, D2H)"}
+    if world == 1 and not args.no_cpu:
+        cpu = cpu_baseline_obj(X, c, args.cpu_seconds)
+    if rank != 0:
+        return
+    line = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic",
+        "config": {"workload": workload_desc(c), "n": n, "d": d, "eps": c.eps, "iters": iters,
+                   "clustering_s": ms / 1e3, "clusters": int(lab.max()) + 1,
+                   "parallelism": f"replicate+own+allgather x{world}" if world > 1 else "single GPU",
+                   "l2": "flushed between steps (256 MiB write); inputs resident in HBM",
+                   "update_share_of_step": upd_share, "update_ms_per_launch": upd_avg,
+                   "launches_per_step": launches / args.steps, "work_counters": work},
+        "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                     "frac": achieved / peak, "traffic": traffic_from_profiles(),
+                     "kernel": "k_update (A6 EGG-update)",
+                     "peak_basis": f"FP32 FMA pipe 2*128 lanes*148 SMs*{fmax:.0f} MHz (sm_max_mhz, MEASURED_PEAKS.json)"},
+        "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk_s,
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+# ---------------------------------------------------- reference arm (oracle)
+def run_reference(args):
+    world, rank, _ = dist_env()
+    if rank != 0:
+        return
+    from paper_conf_edbt_jorgensena23_b200 import datagen
+    c = datagen.make_config(args.config)
+    X = c.generate(args.seed)
+    rate0, m, dt, cores = oracle_rate(X, c.eps, args.cpu_seconds / 2)
+    rng = np.random.default_rng(1)
+    import oracle
+    ts = []
+    for k in range(args.warmup + args.steps):
+        idx = rng.choice(len(X), m, replace=False)
+        t0 = time.perf_counter()
+        oracle.step_sample(X, c.eps, idx)
+        if k >= args.warmup:
+            ts.append(time.perf_counter() - t0)
+    sec = statistics.mean(ts)
+    value = m / sec
+    sample = (f"{m} Eq.1 point-updates per step of {c.name} iteration 1 (each against the full n={c.n:,} state), "
+              f"fp64 C/OpenMP oracle on {cores} threads")
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": sec * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": workload_desc(c), "n": c.n, "d": c.d, "eps": c.eps, "sample_points_per_step": m},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--config", default="C3")
+    ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

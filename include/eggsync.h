@@ -191,6 +191,19 @@ int eggsync_ctx_run(eggsync_ctx *ctx, int32_t max_iters, int32_t *iters_out);
 /* Stream of the context (cudaStream_t). */
 void *eggsync_ctx_stream(eggsync_ctx *ctx);
 
+/* Work counters of the update kernel (for the roofline).
+ * enable = 1: reset the counters and run subsequent updates in the instrumented
+ * variant; 0: back to the plain variant; -1: leave as is.  totals_out (host, 8
+ * int64, may be NULL) receives, before the enable takes effect: [0] (point,cell)
+ * classifications, [1] summary/point accumulations, [2] (point,point) scan tests,
+ * [3] (point,subtree) box tests, [4] fp64 re-decisions, [5] (point,partial cell)
+ * pairs, [6] full-subtree uses, [7] staged cells.  Synchronises. */
+int eggsync_ctx_work(eggsync_ctx *ctx, int32_t enable, int64_t *totals_out);
+
+/* Number of kernel launches this context has issued (CUB's internal launches
+ * counted per pass). */
+int64_t eggsync_ctx_launches(eggsync_ctx *ctx);
+
 #ifdef __cplusplus
 }
 #endif

@@ -124,6 +124,7 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
       {(void**)&c_minorig, sizeof(uint32_t) * cap},
       {(void**)&nbr, sizeof(int32_t) * n},
       {(void**)&lab_final, sizeof(int32_t) * n},
+      {(void**)&work, sizeof(unsigned long long) * 8},
   };
   size_t total = 0;
   for (auto& it : items) total += (it.bytes + 255) & ~size_t(255);
@@ -249,6 +250,7 @@ static int iterate(Workspace& ws, int32_t* synced, int32_t* f1o, int32_t* f2o, i
   if (!ws.built) EGG_TRY(stage_build(ws));
   if (stats) EGG_CUDA(cudaEventRecord(ws.ev[1], ws.stream));
   k_set_flags<<<1, 1, 0, ws.stream>>>(ws.flags, 1, 1);
+  ws.launches++;
   EGG_CUDA(cudaGetLastError());
   EGG_TRY(stage_update(ws, 0, ws.n, nbr_sorted));
   if (stats) EGG_CUDA(cudaEventRecord(ws.ev[2], ws.stream));
@@ -531,6 +533,7 @@ int eggsync_ctx_build(eggsync_ctx* ctx, int32_t* n_cells_out) {
   Workspace& ws = ctx->ws;
   EGG_TRY(stage_build(ws));
   k_set_flags<<<1, 1, 0, ws.stream>>>(ws.flags, 1, 1);
+  ws.launches++;
   EGG_CUDA(cudaGetLastError());
   ws.second_checked = false;
   if (n_cells_out) *n_cells_out = ws.n_cells;
@@ -571,6 +574,7 @@ int eggsync_ctx_pack(eggsync_ctx* ctx, int64_t lo, int64_t cnt, float* buf) {
   const int64_t tot = cnt * ws.d;
   if (tot == 0) return EGGSYNC_OK;
   k_pack<<<(unsigned)((tot + 255) / 256), 256, 0, ws.stream>>>(ws.xs[ws.xcur ^ 1], ws.n, ws.d, lo, cnt, buf);
+  ws.launches++;
   EGG_CUDA(cudaGetLastError());
   return EGGSYNC_OK;
 }
@@ -582,6 +586,7 @@ int eggsync_ctx_unpack(eggsync_ctx* ctx, const float* gathered, int32_t ranks, i
   if (tot == 0) return EGGSYNC_OK;
   k_unpack<<<(unsigned)((tot + 255) / 256), 256, 0, ws.stream>>>(gathered, ws.n, ws.d, ranks, cnt,
                                                                   ws.xs[ws.xcur ^ 1]);
+  ws.launches++;
   EGG_CUDA(cudaGetLastError());
   return EGGSYNC_OK;
 }
@@ -627,5 +632,23 @@ int eggsync_ctx_run(eggsync_ctx* ctx, int32_t max_iters, int32_t* iters_out) {
 }
 
 void* eggsync_ctx_stream(eggsync_ctx* ctx) { return ctx ? (void*)ctx->ws.stream : nullptr; }
+
+int eggsync_ctx_work(eggsync_ctx* ctx, int32_t enable, int64_t* totals_out) {
+  if (!ctx) return EGGSYNC_EINVAL;
+  Workspace& ws = ctx->ws;
+  if (totals_out) {
+    EGG_CUDA(cudaMemcpyAsync(totals_out, ws.work, 8 * sizeof(int64_t), cudaMemcpyDeviceToHost, ws.stream));
+    EGG_CUDA(cudaStreamSynchronize(ws.stream));
+  }
+  if (enable == 1) {
+    EGG_CUDA(cudaMemsetAsync(ws.work, 0, 8 * sizeof(int64_t), ws.stream));
+    ws.count_work = true;
+  } else if (enable == 0) {
+    ws.count_work = false;
+  }
+  return EGGSYNC_OK;
+}
+
+int64_t eggsync_ctx_launches(eggsync_ctx* ctx) { return ctx ? ctx->ws.launches : -1; }
 
 }  // extern "C"

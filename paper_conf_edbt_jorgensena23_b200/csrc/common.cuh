@@ -157,6 +157,9 @@ struct Workspace {
   cudaEvent_t ev[8];
   bool ev_ok = false;
   int sort_skipped = 0;
+  unsigned long long* work = nullptr;  // [8] work counters of the instrumented update
+  bool count_work = false;
+  int64_t launches = 0;  // kernel launches issued on this workspace (CUB internals counted by pass)
 
   int alloc(int64_t n, int d, float eps, int device, cudaStream_t stream);
   void release();

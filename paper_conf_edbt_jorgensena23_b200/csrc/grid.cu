@@ -409,7 +409,14 @@ __global__ void k_scatter_i32(const int32_t* __restrict__ v, const uint32_t* __r
 }
 
 // ===================================================================== hosts
-#define EGG_LAUNCH_CHECK() EGG_CUDA(cudaGetLastError())
+#define EGG_LAUNCH_CHECK() \
+  do {                     \
+    ws.launches++;         \
+    EGG_CUDA(cudaGetLastError()); \
+  } while (0)
+// CUB launches (onesweep radix sort: histogram + exclusive sum + one pass per 8 bits;
+// single-tile sort for small n; scans: init + sweep).
+static inline int cub_sort_launches(int64_t n, int bits) { return n <= 4096 ? 1 : 2 + (bits + 7) / 8; }
 
 int stage_ingest(Workspace& ws, const float* points, bool on_device) {
   const int64_t nd = ws.n * ws.d;
@@ -462,6 +469,7 @@ static int build_d(Workspace& ws) {
       const int wbits = (w < K.nw - 1) ? 64 : (K.keybits - 64 * (K.nw - 1));
       size_t bytes = ws.cub_bytes;
       EGG_CUDA(cub::DeviceRadixSort::SortPairs(ws.cub_tmp, bytes, kbuf, pbuf, (int)n, 0, wbits, st));
+      ws.launches += cub_sort_launches(n, wbits);
     }
     k_gather_state<D><<<blocks_for(n, T), T, 0, st>>>(ws.xs[ws.xcur], ws.orig[ws.ocur], ws.keys, pbuf.Current(),
                                                       n, K.nw, ws.xs[ws.xcur ^ 1], ws.orig[ws.ocur ^ 1],
@@ -479,6 +487,7 @@ static int build_d(Workspace& ws) {
   {
     size_t bytes = ws.cub_bytes;
     EGG_CUDA(cub::DeviceScan::InclusiveSum(ws.cub_tmp, bytes, ws.iscan, ws.cell_of, (int)n, st));
+    ws.launches += 2;
   }
   k_cell_start<<<blocks_for(n, T), T, 0, st>>>(ws.iscan, ws.cell_of, n, K.nw, ws.keys, cap, ws.cell_start,
                                                ws.c_key);
@@ -550,6 +559,7 @@ int stage_labels(Workspace& ws, int32_t* labels_dev) {
   EGG_LAUNCH_CHECK();
   size_t bytes = ws.cub_bytes;
   EGG_CUDA(cub::DeviceScan::ExclusiveSum(ws.cub_tmp, bytes, ws.i_lab, ws.iscan, (int)n, st));
+  ws.launches += 2;
   k_lab_write<<<blocks_for(n, T), T, 0, st>>>(ws.cell_of, ws.orig[ws.ocur], ws.c_minorig, ws.iscan, n, labels_dev);
   EGG_LAUNCH_CHECK();
   return EGGSYNC_OK;

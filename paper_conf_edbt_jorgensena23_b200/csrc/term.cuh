@@ -176,6 +176,7 @@ int run_second_term(Workspace& ws, int64_t lo, int64_t hi) {
   EGG_CUDA(cudaFuncSetAttribute(k_second<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   const int64_t per = 32 * kWarpsPerCta;
   k_second<D><<<(unsigned)((hi - lo + per - 1) / per), kWarpsPerCta * 32, smem, ws.stream>>>(a);
+  ws.launches += 1;
   EGG_CUDA(cudaGetLastError());
   return EGGSYNC_OK;
 }

@@ -49,6 +49,19 @@ struct UpdArgs {
   double e2d;
   int32_t* flags;  // [0] first term AND, [3] error
   int32_t* nbr;    // optional |N(p)| (sorted order)
+  unsigned long long* work;  // optional work counters (CNT variant), see WorkCnt
+};
+
+// Work counters of the instrumented variant (lane-level events, summed per warp).
+struct WorkCnt {
+  long long cls = 0;     // (point, staged cell) classifications
+  long long acc = 0;     // summary / point accumulations (2D adds each)
+  long long scan = 0;    // (point, point) distance tests in partial-cell scans
+  long long node = 0;    // (point, subtree box) tests
+  long long exact = 0;   // fp64 re-decisions inside the error band
+  long long part = 0;    // (point, partial cell) pairs
+  long long nfull = 0;   // full-subtree summary uses
+  long long staged = 0;  // cells staged into shared memory (per warp)
 };
 
 __device__ __forceinline__ float ordf(uint32_t o) {
@@ -89,9 +102,9 @@ struct UpdState {
 };
 
 // Exact point scan of one partial cell for lanes with `pa` (warp-uniform call).
-template <int D>
+template <int D, bool CNT>
 __device__ __forceinline__ void scan_cell(const UpdArgs<D>& a, UpdState<D>& s, bool pa, int32_t c,
-                                       const float* __restrict__ sg) {
+                                          const float* __restrict__ sg, WorkCnt& wc) {
   constexpr int KA = Stage<D>::kA, KB = Stage<D>::kB;
   const int32_t cnt = __float_as_int(sg[KA + KB]);
   const int32_t start = __float_as_int(sg[KA + KB + 1]);
@@ -107,6 +120,7 @@ __device__ __forceinline__ void scan_cell(const UpdArgs<D>& a, UpdState<D>& s, b
   }
   const bool full = pa && maxd <= a.e2f * (1.f - a.rel);
   pa = pa && !full && mind <= a.e2f * (1.f + a.rel);
+  if constexpr (CNT) wc.acc += __popc(__ballot_sync(FULLMASK, full));
   if (__any_sync(FULLMASK, full)) {
     const float f = full ? 1.f : 0.f;
 #pragma unroll
@@ -134,6 +148,11 @@ __device__ __forceinline__ void scan_cell(const UpdArgs<D>& a, UpdState<D>& s, b
     if (__any_sync(FULLMASK, amb)) {
       if (amb) in = exact_d2<D>(qv, s.p) <= a.e2d;
     }
+    if constexpr (CNT) {
+      wc.scan += __popc(__ballot_sync(FULLMASK, pa));
+      wc.exact += __popc(__ballot_sync(FULLMASK, amb));
+      wc.acc += __popc(__ballot_sync(FULLMASK, in));
+    }
     if (__any_sync(FULLMASK, in)) {
       const float f = in ? 1.f : 0.f;
 #pragma unroll
@@ -150,10 +169,10 @@ __device__ __forceinline__ void scan_cell(const UpdArgs<D>& a, UpdState<D>& s, b
 
 // Stage cells [first, first+cnt) (cnt <= 32) into the warp's shared buffer and
 // accumulate them for the lanes in `pm`.
-template <int D>
+template <int D, bool CNT>
 __device__ __forceinline__ void process_cells(const UpdArgs<D>& a, UpdState<D>& s, int32_t first, int32_t cntc,
                                               unsigned pm, float* __restrict__ st,
-                                              const float* __restrict__ ov, int lane) {
+                                              const float* __restrict__ ov, int lane, WorkCnt& wc) {
   constexpr int SF = Stage<D>::kFloats, KA = Stage<D>::kA, KB = Stage<D>::kB;
   constexpr int R = CellRec<D>::kFloats;
   __syncwarp();
@@ -186,6 +205,10 @@ __device__ __forceinline__ void process_cells(const UpdArgs<D>& a, UpdState<D>& 
   }
   __syncwarp();
   const bool act = (pm >> lane) & 1u;
+  if constexpr (CNT) {
+    wc.staged += cntc;
+    wc.cls += (long long)cntc * __popc(pm);
+  }
   for (int g = 0; g < cntc; ++g) {
     const float* __restrict__ sg = st + g * SF;
     float cb[KA];
@@ -202,7 +225,11 @@ __device__ __forceinline__ void process_cells(const UpdArgs<D>& a, UpdState<D>& 
     for (int i = 0; i < D; ++i) acc = fmaf(s.m2p[i], cb[i], acc);
     const bool in = act && acc <= cb[D + 1];
     const bool pa = act && !in && acc <= cb[D + 2];
-    if (__any_sync(FULLMASK, pa)) scan_cell<D>(a, s, pa, first + g, sg);
+    if constexpr (CNT) {
+      wc.part += __popc(__ballot_sync(FULLMASK, pa));
+      wc.acc += __popc(__ballot_sync(FULLMASK, in));
+    }
+    if (__any_sync(FULLMASK, pa)) scan_cell<D, CNT>(a, s, pa, first + g, sg, wc);
     if (__any_sync(FULLMASK, in)) {
       float sb[KB];
 #pragma unroll
@@ -225,7 +252,7 @@ __device__ __forceinline__ void process_cells(const UpdArgs<D>& a, UpdState<D>& 
   s.flush();
 }
 
-template <int D>
+template <int D, bool CNT>
 __global__ void __launch_bounds__(kWarpsPerCta * 32) k_update(const UpdArgs<D> a) {
   constexpr int SF = Stage<D>::kFloats;
   constexpr int BS = ceil4(2 * D);
@@ -274,6 +301,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_update(const UpdArgs<D> a
   s.N = 0;
 
   const float lim_out = a.e2f * (1.f + a.rel), lim_full = a.e2f * (1.f - a.rel);
+  WorkCnt wc;
   int sp = 1;
   if (lane == 0) stk[0] = make_int2(a.nc > 1 ? 0 : (int)kLeafBit, (int)amask);
   __syncwarp();
@@ -284,7 +312,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_update(const UpdArgs<D> a
     const unsigned m = (unsigned)ent.y;
     const bool act = (m >> lane) & 1u;
     if (ent.x & (int)kLeafBit) {
-      process_cells<D>(a, s, ent.x & 0x7fffffff, 1, m, st, ov, lane);
+      process_cells<D, CNT>(a, s, ent.x & 0x7fffffff, 1, m, st, ov, lane, wc);
       continue;
     }
     const int node = ent.x;
@@ -299,6 +327,12 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_update(const UpdArgs<D> a
     }
     const bool full = act && maxd <= lim_full;
     const bool part = act && !full && mind <= lim_out;
+    if constexpr (CNT) {
+      wc.node += __popc(m);
+      const int nf = __popc(__ballot_sync(FULLMASK, full));
+      wc.nfull += nf;
+      wc.acc += nf;
+    }
     if (__any_sync(FULLMASK, full)) {
       if (full) {
         const float* __restrict__ sm = a.t_sum + (int64_t)node * BS;
@@ -314,7 +348,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_update(const UpdArgs<D> a
     if (pm == 0u) continue;
     const int4 meta = a.t_meta[node];
     if (meta.y - meta.x + 1 <= kBucket) {
-      process_cells<D>(a, s, meta.x, meta.y - meta.x + 1, pm, st, ov, lane);
+      process_cells<D, CNT>(a, s, meta.x, meta.y - meta.x + 1, pm, st, ov, lane, wc);
     } else {
       if (sp + 2 > a.stack_len) {  // cannot happen for depth <= key bits; guard anyway
         if (lane == 0) atomicExch(&a.flags[3], 1);
@@ -344,6 +378,18 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_update(const UpdArgs<D> a
     if (a.nbr) a.nbr[j] = s.N;
   }
   if (__any_sync(FULLMASK, !f1) && lane == 0) atomicAnd(&a.flags[0], 0);
+  if constexpr (CNT) {
+    if (lane == 0) {
+      atomicAdd(&a.work[0], (unsigned long long)wc.cls);
+      atomicAdd(&a.work[1], (unsigned long long)wc.acc);
+      atomicAdd(&a.work[2], (unsigned long long)wc.scan);
+      atomicAdd(&a.work[3], (unsigned long long)wc.node);
+      atomicAdd(&a.work[4], (unsigned long long)wc.exact);
+      atomicAdd(&a.work[5], (unsigned long long)wc.part);
+      atomicAdd(&a.work[6], (unsigned long long)wc.nfull);
+      atomicAdd(&a.work[7], (unsigned long long)wc.staged);
+    }
+  }
 }
 
 template <int D>
@@ -375,14 +421,17 @@ int run_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   a.e2d = ws.k.e2;
   a.flags = ws.flags;
   a.nbr = nbr;
+  a.work = ws.count_work ? ws.work : nullptr;
   constexpr int SF = Stage<D>::kFloats;
   constexpr int OV = ceil4(D + 1);
   const size_t smem = (size_t)kWarpsPerCta * (32 * SF + OV) * sizeof(float) +
                       (size_t)kWarpsPerCta * a.stack_len * sizeof(int2);
-  EGG_CUDA(cudaFuncSetAttribute(k_update<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  auto kern = a.work ? k_update<D, true> : k_update<D, false>;
+  EGG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   const int64_t pts_per_cta = 32 * kWarpsPerCta;
   const unsigned grid = (unsigned)((hi - lo + pts_per_cta - 1) / pts_per_cta);
-  k_update<D><<<grid, kWarpsPerCta * 32, smem, ws.stream>>>(a);
+  kern<<<grid, kWarpsPerCta * 32, smem, ws.stream>>>(a);
+  ws.launches += 1;
   EGG_CUDA(cudaGetLastError());
   return EGGSYNC_OK;
 }

@@ -1,0 +1,90 @@
+"""Algorithm 4 over the phase API, single- or multi-rank.
+
+Multi-GPU scheme ("replicate + own + all-gather"):
+every rank holds all n points and builds the identical structure (the build
+is deterministic: Morton keys, stable sort, integer summaries), updates only
+its contiguous range [lo, hi) of the sorted order (Eq.1 is a Jacobi update,
+L68, so ranges are independent given D^t), then the ranks exchange their
+updated ranges with one all-gather (NCCL over NVLink via torch.distributed)
+and AND-reduce the two criterion flags.  The result is bitwise identical to
+one GPU.  torch.distributed is plumbing only; all arithmetic is in the
+library's kernels.
+"""
+from __future__ import annotations
+
+import math
+
+
+class LocalComm:
+    """World size 1: the whole range, no exchange."""
+
+    def __init__(self, n: int):
+        self.rank, self.world, self.lo, self.hi, self.cnt = 0, 1, 0, n, n
+
+    def reduce_min(self, v: int) -> int:
+        return v
+
+    def exchange(self, ctx) -> None:
+        pass
+
+
+class TorchComm:
+    """Rank r owns sorted positions [r*cnt, min(n, (r+1)*cnt)), cnt = ceil(n / world)."""
+
+    def __init__(self, n: int, d: int, device, group=None):
+        import torch
+        import torch.distributed as dist
+        self.dist, self.group = dist, group
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self.cnt = math.ceil(n / self.world)
+        self.lo = min(n, self.rank * self.cnt)
+        self.hi = min(n, self.lo + self.cnt)
+        self.send = torch.empty((d, self.cnt), dtype=torch.float32, device=device)
+        self.recv = torch.empty((self.world, d, self.cnt), dtype=torch.float32, device=device)
+        self.flag = torch.zeros(1, dtype=torch.int32, device=device)
+
+    def reduce_min(self, v: int) -> int:
+        self.flag.fill_(int(v))
+        self.dist.all_reduce(self.flag, op=self.dist.ReduceOp.MIN, group=self.group)
+        return int(self.flag.item())
+
+    def exchange(self, ctx) -> None:
+        ctx.pack_into(self.lo, self.cnt, self.send)
+        self.dist.all_gather_into_tensor(self.recv, self.send, group=self.group)
+        ctx.unpack_from(self.recv, self.world, self.cnt)
+
+
+def run(ctx, comm=None, max_iters: int = 10000, hooks=None):
+    """Iterate until the criterion holds on the state the update read (readings R6/R7).
+
+    ctx   : eggsync.Context (or any object with the same phase methods)
+    comm  : LocalComm / TorchComm (None = LocalComm)
+    hooks : optional object with before_update() / after_update() (timing)
+    Returns (iters, converged, labels).
+    """
+    comm = comm or LocalComm(ctx.n)
+    t, synced, labels = 0, False, None
+    while True:
+        ctx.build()
+        if hooks:
+            hooks.before_update()
+        ctx.update(comm.lo, comm.hi)                      # Alg 3 on the owned range
+        if hooks:
+            hooks.after_update()
+        f1 = comm.reduce_min(ctx.flags()[0])              # first term (Alg 3 l.14-15)
+        f2 = -1
+        if f1 == 1:                                       # Alg 4 l.9-10
+            ctx.second_term(comm.lo, comm.hi)
+            f2 = comm.reduce_min(ctx.flags()[1])
+        synced = f1 == 1 and f2 == 1
+        comm.exchange(ctx)                                # all ranks get D^{t+1}
+        if synced:
+            labels = ctx.labels()                         # cells of the verified state (L256)
+        ctx.advance()
+        t += 1
+        if synced or t >= max_iters:
+            break
+    if not synced:
+        labels = ctx.labels()
+    return t, synced, labels

@@ -25,7 +25,7 @@ SYMBOLS = [
     "eggsync_ctx_load", "eggsync_ctx_build", "eggsync_ctx_update", "eggsync_ctx_second_term",
     "eggsync_ctx_flags", "eggsync_ctx_cur_coords", "eggsync_ctx_next_coords", "eggsync_ctx_pack",
     "eggsync_ctx_unpack", "eggsync_ctx_advance", "eggsync_ctx_labels", "eggsync_ctx_coords",
-    "eggsync_ctx_run", "eggsync_ctx_stream",
+    "eggsync_ctx_run", "eggsync_ctx_stream", "eggsync_ctx_work", "eggsync_ctx_launches",
 ]
 
 
@@ -89,6 +89,8 @@ def lib():
             "eggsync_ctx_coords": ([vp, vp, i32], ctypes.c_int),
             "eggsync_ctx_run": ([vp, i32, vp], ctypes.c_int),
             "eggsync_ctx_stream": ([vp], vp),
+            "eggsync_ctx_work": ([vp, i32, vp], ctypes.c_int),
+            "eggsync_ctx_launches": ([vp], ctypes.c_int64),
         }
         for name, (args, res) in sig.items():
             fn = getattr(L, name)
@@ -244,6 +246,14 @@ class Context:
     def unpack(self, gathered_ptr: int, ranks: int, cnt: int):
         _check(lib().eggsync_ctx_unpack(self.h, ctypes.c_void_p(gathered_ptr), ranks, cnt))
 
+    def pack_into(self, lo: int, cnt: int, tensor):
+        """Next-state columns [lo, lo+cnt) into a CUDA tensor of shape (d, cnt)."""
+        self.pack(lo, cnt, tensor.data_ptr())
+
+    def unpack_from(self, tensor, ranks: int, cnt: int):
+        """Gathered (ranks, d, cnt) CUDA tensor into the next-state buffer."""
+        self.unpack(tensor.data_ptr(), ranks, cnt)
+
     def advance(self):
         _check(lib().eggsync_ctx_advance(self.h))
 
@@ -267,3 +277,14 @@ class Context:
 
     def stream(self) -> int:
         return lib().eggsync_ctx_stream(self.h) or 0
+
+    WORK_KEYS = ("cls", "acc", "scan", "node", "exact", "part", "nfull", "staged")
+
+    def work(self, enable: int = -1):
+        """Read the update's work counters (dict), then set counting on (1) / off (0) / unchanged (-1)."""
+        out = np.zeros(8, np.int64)
+        _check(lib().eggsync_ctx_work(self.h, enable, out.ctypes.data_as(ctypes.c_void_p)))
+        return dict(zip(self.WORK_KEYS, out.tolist()))
+
+    def launches(self) -> int:
+        return int(lib().eggsync_ctx_launches(self.h))
