@@ -155,7 +155,10 @@ def run_ours(args):
     c = datagen.make_config(args.config)
     X = c.generate(args.seed)
     n, d = X.shape
-    stream = torch.cuda.current_stream(dev)
+    # one explicit stream for the library, the L2 flush, the events and the collectives
+    # (the legacy default stream has handle 0, which the library would replace by its own)
+    stream = torch.cuda.Stream(dev)
+    torch.cuda.set_stream(stream)
     Xd = torch.from_numpy(X).to(dev)
     ctx = E.Context(n, d, c.eps, device=local, stream=stream.cuda_stream)
     comm = DR.TorchComm(n, d, dev) if world > 1 else DR.LocalComm(n)

@@ -14,12 +14,12 @@ import sys
 
 HERE = os.path.dirname(os.path.abspath(__file__))
 CSRC = os.path.join(HERE, "csrc")
-OUT = os.path.join(HERE, "libeggsync.so")
-BUILD = os.path.join(HERE, "_build")
+OUT = os.environ.get("EGG_OUT") or os.path.join(HERE, "libeggsync.so")
+BUILD = os.environ.get("EGG_BUILD_DIR") or os.path.join(HERE, "_build")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-O2",
-         "--expt-relaxed-constexpr", "-I", os.path.join(HERE, "..", "include")]
+         "--expt-relaxed-constexpr", "-I", os.path.join(HERE, "..", "include")] + os.environ.get("EGG_NVCC_EXTRA", "").split()
 
 
 def _sources():

@@ -94,6 +94,40 @@ void set_error(const char* fmt, ...);
     if (_rc != EGGSYNC_OK) return _rc; \
   } while (0)
 
+
+// Dimension dispatch (kernels are templated on D = 1..kMaxD).  A development build
+// with -DEGG_DEV_D=<d> instantiates a single dimension (fast rebuilds for tuning).
+#ifdef EGG_DEV_D
+#define EGG_DIM_ENABLED(x) ((x) == EGG_DEV_D)
+#else
+#define EGG_DIM_ENABLED(x) true
+#endif
+#define EGG_CASE_D(Dv, FN, ...)                           \
+  case Dv:                                                \
+    if constexpr (EGG_DIM_ENABLED(Dv)) {                  \
+      return FN<Dv>(__VA_ARGS__);                         \
+    } else {                                              \
+      set_error("d=%d not built (EGG_DEV_D build)", Dv);  \
+      return EGGSYNC_EINVAL;                              \
+    }
+#define EGG_DISPATCH(d, FN, ...)                                                                        \
+  switch (d) {                                                                                          \
+    EGG_CASE_D(1, FN, __VA_ARGS__) EGG_CASE_D(2, FN, __VA_ARGS__) EGG_CASE_D(3, FN, __VA_ARGS__)        \
+    EGG_CASE_D(4, FN, __VA_ARGS__) EGG_CASE_D(5, FN, __VA_ARGS__) EGG_CASE_D(6, FN, __VA_ARGS__)        \
+    EGG_CASE_D(7, FN, __VA_ARGS__) EGG_CASE_D(8, FN, __VA_ARGS__) EGG_CASE_D(9, FN, __VA_ARGS__)        \
+    EGG_CASE_D(10, FN, __VA_ARGS__) EGG_CASE_D(11, FN, __VA_ARGS__) EGG_CASE_D(12, FN, __VA_ARGS__)     \
+    EGG_CASE_D(13, FN, __VA_ARGS__) EGG_CASE_D(14, FN, __VA_ARGS__) EGG_CASE_D(15, FN, __VA_ARGS__)     \
+    EGG_CASE_D(16, FN, __VA_ARGS__) EGG_CASE_D(17, FN, __VA_ARGS__) EGG_CASE_D(18, FN, __VA_ARGS__)     \
+    EGG_CASE_D(19, FN, __VA_ARGS__) EGG_CASE_D(20, FN, __VA_ARGS__) EGG_CASE_D(21, FN, __VA_ARGS__)     \
+    EGG_CASE_D(22, FN, __VA_ARGS__) EGG_CASE_D(23, FN, __VA_ARGS__) EGG_CASE_D(24, FN, __VA_ARGS__)     \
+    EGG_CASE_D(25, FN, __VA_ARGS__) EGG_CASE_D(26, FN, __VA_ARGS__) EGG_CASE_D(27, FN, __VA_ARGS__)     \
+    EGG_CASE_D(28, FN, __VA_ARGS__) EGG_CASE_D(29, FN, __VA_ARGS__) EGG_CASE_D(30, FN, __VA_ARGS__)     \
+    EGG_CASE_D(31, FN, __VA_ARGS__) EGG_CASE_D(32, FN, __VA_ARGS__)                                    \
+    default:                                                                                            \
+      set_error("unsupported d=%d", d);                                                                 \
+      return EGGSYNC_EINVAL;                                                                            \
+  }
+
 // ------------------------------------------------------------------ workspace
 struct Workspace {
   Consts k;

@@ -1,32 +1,47 @@
 // update.cuh -- A6 EGG-update (Algorithm 3; §4.3.2) and
 // A7a first-term flag (Alg 3 l.14-15, L252), templated on the dimension D.
 //
-// For every point p (one lane each, 32 consecutive sorted points per warp):
-//   sum_{q in N_eps(p)} sin(q_i)  and  sum cos(q_i)   (Eq.5)
+// For every point p:
+//   S_i = sum_{q in N_eps(p)} sin(q_i),  C_i = sum_{q in N_eps(p)} cos(q_i)   (Eq.5)
 // split into full and partial pieces (Eq.6):
 //   * subtree of the cell hierarchy entirely inside the eps-ball of p
-//     -> its summary (count, sum sin, sum cos)           [full fast path]
+//     -> its summary (count, sum sin, sum cos)                [full fast path]
 //   * subtree entirely outside -> skipped
-//   * otherwise descend; at <= kBucket cells the cells are staged in shared
-//     memory (origin-shifted to the warp's MBR centre) and classified per lane:
-//     full cell -> cell summary; partial cell -> exact point scan  [boundary scan]
-// then p_i <- p_i + (cos p_i * S_i - sin p_i * C_i) / |N|   (fp64 epilogue)
+//   * otherwise descend; at <= a.bucket cells the cells are staged in shared
+//     memory (origin-shifted to the warp's MBR centre) and classified per
+//     point: full cell -> cell summary; partial cell -> exact point scan
+//                                                              [boundary scan]
+// then p_i <- p_i + (cos p_i * S_i - sin p_i * C_i) / |N|      (fp64 epilogue)
 // and the first term |N_eps(p)| == |cell(p)| is AND-reduced into flags[0].
 //
-// The traversal is a warp "packet": one shared stack of (node, lane mask); a
-// node is visited iff some lane still needs it, and every lane classifies it
-// against its own point, so noise points and cluster points in one warp do
-// not inflate each other's work.
+// Execution: one warp owns 64 consecutive sorted points (2 per lane: two
+// independent dependency chains per lane, and every staged cell read from
+// shared memory is used twice).  The traversal is a warp "packet": one shared
+// stack of (node, 64-bit point mask); a node is visited iff some point still
+// needs it, and every point classifies it against itself, so noise points and
+// cluster points in one warp do not inflate each other's work.
 //
-// Exactness: every "full"/"out" decision carries a proven fp32 error margin;
-// point pairs inside the margin are re-decided in fp64 exactly as the oracle's
-// sum_i (q_i - p_i)^2 <= eps^2 (dimension order, no FMA).
+// Arithmetic: the squared distance to a staged cell uses the expanded form
+// |q|^2 + |c'|^2 - 2 q.c' in the warp's shifted frame (D FMAs, two chains);
+// sums are accumulated in fp32 per bucket and flushed into fp64 masters kept
+// in shared memory.  Every "full"/"out" decision carries a proven fp32 error
+// margin; point pairs inside the margin are re-decided in fp64 exactly as the
+// oracle's sum_i (q_i - p_i)^2 <= eps^2 (dimension order, no FMA).
 #pragma once
 #include "common.cuh"
 
 namespace egg {
 
 #define FULLMASK 0xffffffffu
+#ifndef EGG_UPD_BUCKET_SPARSE
+#define EGG_UPD_BUCKET_SPARSE 256  // cells mostly singletons (early iterations)
+#define EGG_UPD_BUCKET_DENSE 64    // dense cells: box pruning pays
+#endif
+#ifndef EGG_UPD_MINB
+#define EGG_UPD_MINB 1
+#endif
+constexpr int kP = 2;                        // points per lane
+// a subtree of <= a.bucket cells is processed cell by cell (chosen per launch, run_update)
 
 template <int D>
 struct UpdArgs {
@@ -44,7 +59,7 @@ struct UpdArgs {
   const float* __restrict__ t_sum;
   const int32_t* __restrict__ t_cnt;
   int64_t n, cap, lo, hi;
-  int32_t nc, stack_len;
+  int32_t nc, stack_len, bucket;
   float e, e2f, rel;
   double e2d;
   int32_t* flags;  // [0] first term AND, [3] error
@@ -52,7 +67,7 @@ struct UpdArgs {
   unsigned long long* work;  // optional work counters (CNT variant), see WorkCnt
 };
 
-// Work counters of the instrumented variant (lane-level events, summed per warp).
+// Work counters of the instrumented variant (point-level events, summed per warp).
 struct WorkCnt {
   long long cls = 0;     // (point, staged cell) classifications
   long long acc = 0;     // summary / point accumulations (2D adds each)
@@ -81,39 +96,60 @@ __device__ __forceinline__ double exact_d2(const float* q, const float* p) {
   return s;
 }
 
-template <int D>
-struct UpdState {
-  float p[D];    // the point
-  float m2p[D];  // -2 (p - o)
-  float pp;      // |p - o|^2
-  float S[D], C[D];    // fp32 chunk accumulators
-  double Sd[D], Cd[D]; // fp64 masters
-  int N;               // |N_eps(p)|
+__device__ __forceinline__ int popc64(unsigned long long m) { return __popcll(m); }
 
-  __device__ __forceinline__ void flush() {
-#pragma unroll
-    for (int i = 0; i < D; ++i) {
-      Sd[i] += (double)S[i];
-      Cd[i] += (double)C[i];
-      S[i] = 0.f;
-      C[i] = 0.f;
-    }
+// Shared-memory layout of one warp (floats unless noted).
+template <int D>
+struct WarpSmem {
+  static constexpr int SF = Stage<D>::kFloats;
+  static constexpr int OV = ceil4(D + 4);  // o[D], Bw, pad
+  static constexpr int kStageFloats = 32 * SF;
+  static constexpr int kMasterDoubles = kP * 2 * D * 32;
+  __host__ __device__ static size_t bytes(int stack_len) {
+    return (size_t)(kStageFloats + OV) * 4 + (size_t)kMasterDoubles * 8 + (size_t)stack_len * 16;
   }
 };
 
-// Exact point scan of one partial cell for lanes with `pa` (warp-uniform call).
+template <int D>
+struct Lane {
+  float q[kP][D];  // p - o (shifted point)
+  float pp[kP];    // |q|^2
+  float S[kP][D], C[kP][D];  // fp32 chunk accumulators
+  int N[kP];       // |N_eps(p)|
+  bool valid[kP];
+  int64_t j[kP];   // sorted position
+};
+
+template <int D>
+__device__ __forceinline__ void flush(Lane<D>& L, int k, double* __restrict__ mst, int lane) {
+#pragma unroll
+  for (int i = 0; i < D; ++i) {
+    double* ms = mst + ((k * 2 * D + i) * 32 + lane);
+    double* mc = mst + ((k * 2 * D + D + i) * 32 + lane);
+    *ms += (double)L.S[k][i];
+    *mc += (double)L.C[k][i];
+    L.S[k][i] = 0.f;
+    L.C[k][i] = 0.f;
+  }
+}
+
+// Exact point scan of one partial cell for point k of the lanes with `pa` (warp-uniform call).
 template <int D, bool CNT>
-__device__ __forceinline__ void scan_cell(const UpdArgs<D>& a, UpdState<D>& s, bool pa, int32_t c,
-                                          const float* __restrict__ sg, WorkCnt& wc) {
+__device__ __forceinline__ void scan_cell(const UpdArgs<D>& a, Lane<D>& L, int k, bool pa, int32_t c,
+                                          const float* __restrict__ sg, double* __restrict__ mst, int lane,
+                                          WorkCnt& wc) {
   constexpr int KA = Stage<D>::kA, KB = Stage<D>::kB;
   const int32_t cnt = __float_as_int(sg[KA + KB]);
   const int32_t start = __float_as_int(sg[KA + KB + 1]);
+  float p[D];  // the exact point (the shifted copy is not exact)
+#pragma unroll
+  for (int i = 0; i < D; ++i) p[i] = L.valid[k] ? a.xs[(int64_t)i * a.n + L.j[k]] : 0.f;
   // refine with the exact MBR of the cell (fp32 + margin)
   float mind = 0.f, maxd = 0.f;
 #pragma unroll
   for (int i = 0; i < D; ++i) {
     const float l = ordf(a.c_lo[(int64_t)i * a.cap + c]), h = ordf(a.c_hi[(int64_t)i * a.cap + c]);
-    const float dl = l - s.p[i], dh = s.p[i] - h;
+    const float dl = l - p[i], dh = p[i] - h;
     const float mn = fmaxf(fmaxf(dl, dh), 0.f), mx = fmaxf(-dl, -dh);
     mind = fmaf(mn, mn, mind);
     maxd = fmaf(mx, mx, maxd);
@@ -125,28 +161,28 @@ __device__ __forceinline__ void scan_cell(const UpdArgs<D>& a, UpdState<D>& s, b
     const float f = full ? 1.f : 0.f;
 #pragma unroll
     for (int i = 0; i < D; ++i) {
-      s.S[i] = fmaf(f, sg[KA + i], s.S[i]);
-      s.C[i] = fmaf(f, sg[KA + D + i], s.C[i]);
+      L.S[k][i] = fmaf(f, sg[KA + i], L.S[k][i]);
+      L.C[k][i] = fmaf(f, sg[KA + D + i], L.C[k][i]);
     }
-    s.N += full ? cnt : 0;
+    L.N[k] += full ? cnt : 0;
   }
   if (!__any_sync(FULLMASK, pa)) return;
-  s.flush();
+  flush(L, k, mst, lane);
   const float lim_in = a.e2f * (1.f - a.rel), lim_out = a.e2f * (1.f + a.rel);
-  for (int32_t k = 0; k < cnt; ++k) {
-    const int64_t q = start + k;
+  for (int32_t t = 0; t < cnt; ++t) {
+    const int64_t q = start + t;
     float qv[D];
     float d2 = 0.f;
 #pragma unroll
     for (int i = 0; i < D; ++i) {
       qv[i] = a.xs[(int64_t)i * a.n + q];
-      const float t = qv[i] - s.p[i];
-      d2 = fmaf(t, t, d2);
+      const float u = qv[i] - p[i];
+      d2 = fmaf(u, u, d2);
     }
     bool in = pa && d2 <= lim_in;
     const bool amb = pa && !in && d2 <= lim_out;
     if (__any_sync(FULLMASK, amb)) {
-      if (amb) in = exact_d2<D>(qv, s.p) <= a.e2d;
+      if (amb) in = exact_d2<D>(qv, p) <= a.e2d;
     }
     if constexpr (CNT) {
       wc.scan += __popc(__ballot_sync(FULLMASK, pa));
@@ -157,22 +193,23 @@ __device__ __forceinline__ void scan_cell(const UpdArgs<D>& a, UpdState<D>& s, b
       const float f = in ? 1.f : 0.f;
 #pragma unroll
       for (int i = 0; i < D; ++i) {
-        s.S[i] = fmaf(f, a.sn[(int64_t)i * a.n + q], s.S[i]);
-        s.C[i] = fmaf(f, a.cs[(int64_t)i * a.n + q], s.C[i]);
+        L.S[k][i] = fmaf(f, a.sn[(int64_t)i * a.n + q], L.S[k][i]);
+        L.C[k][i] = fmaf(f, a.cs[(int64_t)i * a.n + q], L.C[k][i]);
       }
-      s.N += in ? 1 : 0;
+      L.N[k] += in ? 1 : 0;
     }
-    if ((k & 31) == 31) s.flush();
+    if ((t & 31) == 31) flush(L, k, mst, lane);
   }
-  s.flush();
+  flush(L, k, mst, lane);
 }
 
-// Stage cells [first, first+cnt) (cnt <= 32) into the warp's shared buffer and
-// accumulate them for the lanes in `pm`.
+// Stage cells [first, first+cntc) (cntc <= 32) into the warp's shared buffer and
+// accumulate them for the points in `pm` (bit k*32+lane = point k of lane).
 template <int D, bool CNT>
-__device__ __forceinline__ void process_cells(const UpdArgs<D>& a, UpdState<D>& s, int32_t first, int32_t cntc,
-                                              unsigned pm, float* __restrict__ st,
-                                              const float* __restrict__ ov, int lane, WorkCnt& wc) {
+__device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int32_t first, int32_t cntc,
+                                            unsigned long long pm, float* __restrict__ st,
+                                            const float* __restrict__ ov, double* __restrict__ mst,
+                                            int lane, WorkCnt& wc) {
   constexpr int SF = Stage<D>::kFloats, KA = Stage<D>::kA, KB = Stage<D>::kB;
   constexpr int R = CellRec<D>::kFloats;
   __syncwarp();
@@ -184,7 +221,7 @@ __device__ __forceinline__ void process_cells(const UpdArgs<D>& a, UpdState<D>& 
 #pragma unroll
     for (int i = 0; i < D; ++i) {
       const float t = r[i] - ov[i];
-      dst[i] = t;
+      dst[i] = -2.f * t;
       cc = fmaf(t, t, cc);
     }
     const float rad = r[D];
@@ -204,33 +241,62 @@ __device__ __forceinline__ void process_cells(const UpdArgs<D>& a, UpdState<D>& 
     dst[KA + KB + 1] = r[D + 2];  // start bits
   }
   __syncwarp();
-  const bool act = (pm >> lane) & 1u;
+  bool act[kP];
+#pragma unroll
+  for (int k = 0; k < kP; ++k) act[k] = (pm >> (k * 32 + lane)) & 1ull;
   if constexpr (CNT) {
     wc.staged += cntc;
-    wc.cls += (long long)cntc * __popc(pm);
+    wc.cls += (long long)cntc * popc64(pm);
   }
-  for (int g = 0; g < cntc; ++g) {
-    const float* __restrict__ sg = st + g * SF;
-    float cb[KA];
+  const float* __restrict__ sg = st;
+  float cb[KA];  // A part of the current cell; the next cell's is loaded one iteration ahead
 #pragma unroll
-    for (int q = 0; q < KA / 4; ++q) {
-      const float4 v = reinterpret_cast<const float4*>(sg)[q];
-      cb[4 * q] = v.x;
-      cb[4 * q + 1] = v.y;
-      cb[4 * q + 2] = v.z;
-      cb[4 * q + 3] = v.w;
+  for (int q = 0; q < KA / 4; ++q) {
+    const float4 v = reinterpret_cast<const float4*>(sg)[q];
+    cb[4 * q] = v.x;
+    cb[4 * q + 1] = v.y;
+    cb[4 * q + 2] = v.z;
+    cb[4 * q + 3] = v.w;
+  }
+  for (int g = 0; g < cntc; ++g, sg += SF) {
+    bool in[kP], pa[kP];
+    bool any_pa = false, any_in = false;
+#pragma unroll
+    for (int k = 0; k < kP; ++k) {
+      float a0 = L.pp[k] + cb[D], a1 = 0.f;
+#pragma unroll
+      for (int i = 0; i < D; i += 2) a0 = fmaf(L.q[k][i], cb[i], a0);
+#pragma unroll
+      for (int i = 1; i < D; i += 2) a1 = fmaf(L.q[k][i], cb[i], a1);
+      const float d2 = a0 + a1;
+      in[k] = act[k] && d2 <= cb[D + 1];
+      pa[k] = act[k] && !in[k] && d2 <= cb[D + 2];
+      any_pa |= pa[k];
+      any_in |= in[k];
     }
-    float acc = s.pp + cb[D];
+    if (g + 1 < cntc) {  // software pipelining: next cell's A part
 #pragma unroll
-    for (int i = 0; i < D; ++i) acc = fmaf(s.m2p[i], cb[i], acc);
-    const bool in = act && acc <= cb[D + 1];
-    const bool pa = act && !in && acc <= cb[D + 2];
+      for (int q = 0; q < KA / 4; ++q) {
+        const float4 v = reinterpret_cast<const float4*>(sg + SF)[q];
+        cb[4 * q] = v.x;
+        cb[4 * q + 1] = v.y;
+        cb[4 * q + 2] = v.z;
+        cb[4 * q + 3] = v.w;
+      }
+    }
     if constexpr (CNT) {
-      wc.part += __popc(__ballot_sync(FULLMASK, pa));
-      wc.acc += __popc(__ballot_sync(FULLMASK, in));
+#pragma unroll
+      for (int k = 0; k < kP; ++k) {
+        wc.part += __popc(__ballot_sync(FULLMASK, pa[k]));
+        wc.acc += __popc(__ballot_sync(FULLMASK, in[k]));
+      }
     }
-    if (__any_sync(FULLMASK, pa)) scan_cell<D, CNT>(a, s, pa, first + g, sg, wc);
-    if (__any_sync(FULLMASK, in)) {
+    if (__any_sync(FULLMASK, any_pa)) {
+#pragma unroll
+      for (int k = 0; k < kP; ++k)
+        if (__any_sync(FULLMASK, pa[k])) scan_cell<D, CNT>(a, L, k, pa[k], first + g, sg, mst, lane, wc);
+    }
+    if (__any_sync(FULLMASK, any_in)) {
       float sb[KB];
 #pragma unroll
       for (int q = 0; q < KB / 4; ++q) {
@@ -240,40 +306,72 @@ __device__ __forceinline__ void process_cells(const UpdArgs<D>& a, UpdState<D>& 
         sb[4 * q + 2] = v.z;
         sb[4 * q + 3] = v.w;
       }
-      const float f = in ? 1.f : 0.f;
+      const int cg = __float_as_int(sg[KA + KB]);
 #pragma unroll
-      for (int i = 0; i < D; ++i) {
-        s.S[i] = fmaf(f, sb[i], s.S[i]);
-        s.C[i] = fmaf(f, sb[D + i], s.C[i]);
+      for (int k = 0; k < kP; ++k) {
+        const float f = in[k] ? 1.f : 0.f;
+#pragma unroll
+        for (int i = 0; i < D; ++i) {
+          L.S[k][i] = fmaf(f, sb[i], L.S[k][i]);
+          L.C[k][i] = fmaf(f, sb[D + i], L.C[k][i]);
+        }
+        L.N[k] += in[k] ? cg : 0;
       }
-      s.N += in ? __float_as_int(sg[KA + KB]) : 0;
     }
   }
-  s.flush();
+}
+
+// A bucket of <= a.bucket consecutive cells: staged and processed 32 at a time,
+// one fp32 -> fp64 flush per bucket (a chunk of at most a.bucket summaries).
+template <int D, bool CNT>
+__device__ __forceinline__ void process_cells(const UpdArgs<D>& a, Lane<D>& L, int32_t first, int32_t cntc,
+                                              unsigned long long pm, float* __restrict__ st,
+                                              const float* __restrict__ ov, double* __restrict__ mst,
+                                              int lane, WorkCnt& wc) {
+  for (int32_t r = 0; r < cntc; r += 32)
+    stage_round<D, CNT>(a, L, first + r, min(32, cntc - r), pm, st, ov, mst, lane, wc);
+#pragma unroll
+  for (int k = 0; k < kP; ++k) flush(L, k, mst, lane);
 }
 
 template <int D, bool CNT>
-__global__ void __launch_bounds__(kWarpsPerCta * 32) k_update(const UpdArgs<D> a) {
-  constexpr int SF = Stage<D>::kFloats;
+__global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(const UpdArgs<D> a) {
+  using W = WarpSmem<D>;
   constexpr int BS = ceil4(2 * D);
-  constexpr int OV = ceil4(D + 1);
   extern __shared__ __align__(16) float smem[];
   const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  float* st = smem + wid * 32 * SF;
-  float* ov = smem + kWarpsPerCta * 32 * SF + wid * OV;
-  int2* stk = reinterpret_cast<int2*>(smem + kWarpsPerCta * (32 * SF + OV)) + wid * a.stack_len;
+  // per-warp regions: [stage+ov floats][masters doubles][stack int4]
+  char* wbase = reinterpret_cast<char*>(smem) + (size_t)wid * W::bytes(a.stack_len);
+  float* st = reinterpret_cast<float*>(wbase);
+  float* ov = st + W::kStageFloats;
+  double* mst = reinterpret_cast<double*>(wbase + (size_t)(W::kStageFloats + W::OV) * 4);
+  int4* stk = reinterpret_cast<int4*>(wbase + (size_t)(W::kStageFloats + W::OV) * 4 + (size_t)W::kMasterDoubles * 8);
 
-  const int64_t j = a.lo + ((int64_t)blockIdx.x * kWarpsPerCta + wid) * 32 + lane;
-  const bool valid = j < a.hi;
-  const unsigned amask = __ballot_sync(FULLMASK, valid);
-  if (amask == 0u) return;
+  const int64_t base = a.lo + ((int64_t)blockIdx.x * kWarpsPerCta + wid) * (32 * kP);
+  Lane<D> L;
+  unsigned long long amask = 0ull;
+#pragma unroll
+  for (int k = 0; k < kP; ++k) {
+    L.j[k] = base + k * 32 + lane;
+    L.valid[k] = L.j[k] < a.hi;
+    amask |= (unsigned long long)__ballot_sync(FULLMASK, L.valid[k]) << (32 * k);
+  }
+  if (amask == 0ull) return;
 
-  UpdState<D> s;
-  // warp MBR centre o (origin for the expanded distance form)
+  // warp MBR centre o: origin of the shifted frame
+  float Rw = 0.f;
 #pragma unroll
   for (int i = 0; i < D; ++i) {
-    s.p[i] = valid ? a.xs[(int64_t)i * a.n + j] : 0.f;
-    float l = valid ? s.p[i] : 3.0e38f, h = valid ? s.p[i] : -3.0e38f;
+    float x[kP];
+    float l = 3.0e38f, h = -3.0e38f;
+#pragma unroll
+    for (int k = 0; k < kP; ++k) {
+      x[k] = L.valid[k] ? a.xs[(int64_t)i * a.n + L.j[k]] : 0.f;
+      if (L.valid[k]) {
+        l = fminf(l, x[k]);
+        h = fmaxf(h, x[k]);
+      }
+    }
 #pragma unroll
     for (int off = 16; off > 0; off >>= 1) {
       l = fminf(l, __shfl_xor_sync(FULLMASK, l, off));
@@ -281,101 +379,150 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_update(const UpdArgs<D> a
     }
     const float o = 0.5f * (l + h);
     if (lane == 0) ov[i] = o;
-    const float t = s.p[i] - o;
-    s.m2p[i] = -2.f * t;
-  }
-  s.pp = 0.f;
 #pragma unroll
-  for (int i = 0; i < D; ++i) s.pp = fmaf(0.5f * s.m2p[i], 0.5f * s.m2p[i], s.pp);
-  {
-    float b = valid ? s.pp : 0.f;
+    for (int k = 0; k < kP; ++k) {
+      L.q[k][i] = L.valid[k] ? x[k] - o : 0.f;
+      Rw = fmaxf(Rw, fabsf(L.q[k][i]));
+    }
+  }
+  float Bw = 0.f;
 #pragma unroll
-    for (int off = 16; off > 0; off >>= 1) b = fmaxf(b, __shfl_xor_sync(FULLMASK, b, off));
-    if (lane == 0) ov[D] = b;
+  for (int k = 0; k < kP; ++k) {
+    float pp = 0.f;
+#pragma unroll
+    for (int i = 0; i < D; ++i) pp = fmaf(L.q[k][i], L.q[k][i], pp);
+    asm volatile("" : "+f"(pp));  // keep it in a register (no rematerialisation in the hot loop)
+    L.pp[k] = pp;
+    Bw = fmaxf(Bw, pp);
+#pragma unroll
+    for (int i = 0; i < D; ++i) {
+      L.S[k][i] = 0.f;
+      L.C[k][i] = 0.f;
+    }
+    L.N[k] = 0;
   }
 #pragma unroll
-  for (int i = 0; i < D; ++i) {
-    s.S[i] = s.C[i] = 0.f;
-    s.Sd[i] = s.Cd[i] = 0.0;
+  for (int off = 16; off > 0; off >>= 1) {
+    Bw = fmaxf(Bw, __shfl_xor_sync(FULLMASK, Bw, off));
+    Rw = fmaxf(Rw, __shfl_xor_sync(FULLMASK, Rw, off));
   }
-  s.N = 0;
+  // subtree-box limits in the shifted frame: the rounding of q = fl(p - o) and
+  // box' = fl(box - o) moves each per-dimension distance by <= 2u(|t| + Rw)
+  const float slack = 2.5f * kU * sqrtf((float)D) * Rw;
+  const float nlo = a.e * (1.f + 4.f * kU) + slack;
+  const float nfu = fmaxf(a.e * (1.f - 4.f * kU) - slack, 0.f);
+  const float lim_out = nlo * nlo * (1.f + (float)(2 * D + 8) * kU);
+  const float lim_full = nfu * nfu * (1.f - (float)(2 * D + 8) * kU);
+  if (lane == 0) ov[D] = Bw;
+  for (int t = lane; t < W::kMasterDoubles; t += 32) mst[t] = 0.0;
+  __syncwarp();
 
-  const float lim_out = a.e2f * (1.f + a.rel), lim_full = a.e2f * (1.f - a.rel);
   WorkCnt wc;
   int sp = 1;
-  if (lane == 0) stk[0] = make_int2(a.nc > 1 ? 0 : (int)kLeafBit, (int)amask);
+  if (lane == 0)
+    stk[0] = make_int4(a.nc > 1 ? 0 : (int)kLeafBit, (int)(uint32_t)amask, (int)(uint32_t)(amask >> 32), 0);
   __syncwarp();
   while (sp > 0) {
     --sp;
-    const int2 ent = stk[sp];
+    const int4 ent = stk[sp];
     __syncwarp();
-    const unsigned m = (unsigned)ent.y;
-    const bool act = (m >> lane) & 1u;
+    const unsigned long long m = (unsigned long long)(uint32_t)ent.y | ((unsigned long long)(uint32_t)ent.z << 32);
     if (ent.x & (int)kLeafBit) {
-      process_cells<D, CNT>(a, s, ent.x & 0x7fffffff, 1, m, st, ov, lane, wc);
+      process_cells<D, CNT>(a, L, ent.x & 0x7fffffff, 1, m, st, ov, mst, lane, wc);
       continue;
     }
     const int node = ent.x;
     const float* __restrict__ bx = a.t_box + (int64_t)node * BS;
-    float mind = 0.f, maxd = 0.f;
+    float lo[D], hi[D];
 #pragma unroll
     for (int i = 0; i < D; ++i) {
-      const float dl = bx[i] - s.p[i], dh = s.p[i] - bx[D + i];
-      const float mn = fmaxf(fmaxf(dl, dh), 0.f), mx = fmaxf(-dl, -dh);
-      mind = fmaf(mn, mn, mind);
-      maxd = fmaf(mx, mx, maxd);
+      lo[i] = bx[i] - ov[i];
+      hi[i] = bx[D + i] - ov[i];
     }
-    const bool full = act && maxd <= lim_full;
-    const bool part = act && !full && mind <= lim_out;
-    if constexpr (CNT) {
-      wc.node += __popc(m);
-      const int nf = __popc(__ballot_sync(FULLMASK, full));
-      wc.nfull += nf;
-      wc.acc += nf;
-    }
-    if (__any_sync(FULLMASK, full)) {
-      if (full) {
-        const float* __restrict__ sm = a.t_sum + (int64_t)node * BS;
+    bool full[kP], part[kP];
+    bool any_full = false;
 #pragma unroll
-        for (int i = 0; i < D; ++i) {
-          s.Sd[i] += (double)sm[i];
-          s.Cd[i] += (double)sm[D + i];
+    for (int k = 0; k < kP; ++k) {
+      const bool act = (m >> (k * 32 + lane)) & 1ull;
+      float m0 = 0.f, m1 = 0.f, x0 = 0.f, x1 = 0.f;
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        const float dl = lo[i] - L.q[k][i], dh = L.q[k][i] - hi[i];
+        const float mn = fmaxf(fmaxf(dl, dh), 0.f), mx = fmaxf(-dl, -dh);
+        if (i & 1) {
+          m1 = fmaf(mn, mn, m1);
+          x1 = fmaf(mx, mx, x1);
+        } else {
+          m0 = fmaf(mn, mn, m0);
+          x0 = fmaf(mx, mx, x0);
         }
-        s.N += a.t_cnt[node];
+      }
+      full[k] = act && (x0 + x1) <= lim_full;
+      part[k] = act && !full[k] && (m0 + m1) <= lim_out;
+      any_full |= full[k];
+    }
+    if constexpr (CNT) {
+      wc.node += popc64(m);
+#pragma unroll
+      for (int k = 0; k < kP; ++k) {
+        const int nf = __popc(__ballot_sync(FULLMASK, full[k]));
+        wc.nfull += nf;
+        wc.acc += nf;
       }
     }
-    const unsigned pm = __ballot_sync(FULLMASK, part);
-    if (pm == 0u) continue;
+    if (__any_sync(FULLMASK, any_full)) {
+      const float* __restrict__ sm = a.t_sum + (int64_t)node * BS;
+      const int cnt = a.t_cnt[node];
+#pragma unroll
+      for (int k = 0; k < kP; ++k) {
+        if (full[k]) {
+#pragma unroll
+          for (int i = 0; i < D; ++i) {
+            mst[(k * 2 * D + i) * 32 + lane] += (double)sm[i];
+            mst[(k * 2 * D + D + i) * 32 + lane] += (double)sm[D + i];
+          }
+          L.N[k] += cnt;
+        }
+      }
+    }
+    unsigned long long pm = 0ull;
+#pragma unroll
+    for (int k = 0; k < kP; ++k) pm |= (unsigned long long)__ballot_sync(FULLMASK, part[k]) << (32 * k);
+    if (pm == 0ull) continue;
     const int4 meta = a.t_meta[node];
-    if (meta.y - meta.x + 1 <= kBucket) {
-      process_cells<D, CNT>(a, s, meta.x, meta.y - meta.x + 1, pm, st, ov, lane, wc);
+    if (meta.y - meta.x + 1 <= a.bucket) {
+      process_cells<D, CNT>(a, L, meta.x, meta.y - meta.x + 1, pm, st, ov, mst, lane, wc);
     } else {
       if (sp + 2 > a.stack_len) {  // cannot happen for depth <= key bits; guard anyway
         if (lane == 0) atomicExch(&a.flags[3], 1);
         break;
       }
       if (lane == 0) {
-        stk[sp] = make_int2(meta.w, (int)pm);
-        stk[sp + 1] = make_int2(meta.z, (int)pm);
+        stk[sp] = make_int4(meta.w, (int)(uint32_t)pm, (int)(uint32_t)(pm >> 32), 0);
+        stk[sp + 1] = make_int4(meta.z, (int)(uint32_t)pm, (int)(uint32_t)(pm >> 32), 0);
       }
       sp += 2;
       __syncwarp();
     }
   }
-  s.flush();
   bool f1 = true;
-  if (valid) {
-    const double inv = 1.0 / (double)s.N;
 #pragma unroll
-    for (int i = 0; i < D; ++i) {
-      double sx, cx;
-      const double x = (double)s.p[i];
-      sincos(x, &sx, &cx);
-      const double xn = x + (cx * s.Sd[i] - sx * s.Cd[i]) * inv;  // Eq.5
-      a.xs_next[(int64_t)i * a.n + j] = fminf(fmaxf((float)xn, 0.f), 1.f);
+  for (int k = 0; k < kP; ++k) {
+    flush(L, k, mst, lane);
+    if (L.valid[k]) {
+      const double inv = 1.0 / (double)L.N[k];
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        double sx, cx;
+        const double x = (double)a.xs[(int64_t)i * a.n + L.j[k]];
+        sincos(x, &sx, &cx);
+        const double Sd = mst[(k * 2 * D + i) * 32 + lane], Cd = mst[(k * 2 * D + D + i) * 32 + lane];
+        const double xn = x + (cx * Sd - sx * Cd) * inv;  // Eq.5
+        a.xs_next[(int64_t)i * a.n + L.j[k]] = fminf(fmaxf((float)xn, 0.f), 1.f);
+      }
+      f1 = f1 && (L.N[k] == a.c_cnt[a.cell_of[L.j[k]]]);  // Alg 3 l.14-15 (L248)
+      if (a.nbr) a.nbr[L.j[k]] = L.N[k];
     }
-    f1 = s.N == a.c_cnt[a.cell_of[j]];  // Alg 3 l.14-15 (L248)
-    if (a.nbr) a.nbr[j] = s.N;
   }
   if (__any_sync(FULLMASK, !f1) && lane == 0) atomicAnd(&a.flags[0], 0);
   if constexpr (CNT) {
@@ -415,6 +562,9 @@ int run_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   a.hi = hi;
   a.nc = ws.n_cells;
   a.stack_len = ws.k.keybits + 4;
+  // mostly-singleton cells (early iterations): subtree boxes rarely prune or cover, so
+  // process bigger buckets; dense cells: descend further and let box tests prune / cover
+  a.bucket = (int64_t)ws.n_cells * 2 > ws.n ? EGG_UPD_BUCKET_SPARSE : EGG_UPD_BUCKET_DENSE;
   a.e = ws.k.ef;
   a.e2f = ws.k.e2f;
   a.rel = ws.k.rel;
@@ -422,13 +572,12 @@ int run_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   a.flags = ws.flags;
   a.nbr = nbr;
   a.work = ws.count_work ? ws.work : nullptr;
-  constexpr int SF = Stage<D>::kFloats;
-  constexpr int OV = ceil4(D + 1);
-  const size_t smem = (size_t)kWarpsPerCta * (32 * SF + OV) * sizeof(float) +
-                      (size_t)kWarpsPerCta * a.stack_len * sizeof(int2);
+  const size_t smem = (size_t)kWarpsPerCta * WarpSmem<D>::bytes(a.stack_len);
   auto kern = a.work ? k_update<D, true> : k_update<D, false>;
   EGG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
-  const int64_t pts_per_cta = 32 * kWarpsPerCta;
+  // all of the 228 KB unified L1/shared to shared memory: occupancy is shared-memory bound
+  EGG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
+  const int64_t pts_per_cta = 32 * kP * kWarpsPerCta;
   const unsigned grid = (unsigned)((hi - lo + pts_per_cta - 1) / pts_per_cta);
   kern<<<grid, kWarpsPerCta * 32, smem, ws.stream>>>(a);
   ws.launches += 1;

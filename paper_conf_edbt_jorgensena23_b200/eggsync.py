@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libeggsync.so")
+LIB_PATH = os.environ.get("EGGSYNC_LIB") or os.path.join(_HERE, "libeggsync.so")
 
 OK, NOT_CONVERGED, EINVAL, EDOMAIN, ENOMEM, ECUDA, ENCCL = 0, 1, -1, -2, -3, -4, -5
 MAX_D = 32
