@@ -41,7 +41,8 @@ class TorchComm:
         self.lo = min(n, self.rank * self.cnt)
         self.hi = min(n, self.lo + self.cnt)
         self.send = torch.empty((d, self.cnt), dtype=torch.float32, device=device)
-        self.recv = torch.empty((self.world, d, self.cnt), dtype=torch.float32, device=device)
+        # concatenated layout (world*d, cnt) == stacked (world, d, cnt) in memory (gloo needs the former)
+        self.recv = torch.empty((self.world * d, self.cnt), dtype=torch.float32, device=device)
         self.flag = torch.zeros(1, dtype=torch.int32, device=device)
 
     def reduce_min(self, v: int) -> int:
@@ -52,7 +53,7 @@ class TorchComm:
     def exchange(self, ctx) -> None:
         ctx.pack_into(self.lo, self.cnt, self.send)
         self.dist.all_gather_into_tensor(self.recv, self.send, group=self.group)
-        ctx.unpack_from(self.recv, self.world, self.cnt)
+        ctx.unpack_from(self.recv.view(self.world, -1, self.cnt), self.world, self.cnt)
 
 
 def run(ctx, comm=None, max_iters: int = 10000, hooks=None):

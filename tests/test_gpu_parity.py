@@ -201,3 +201,59 @@ def test_c3_cluster_terminal_property(c3):
     assert np.array_equal(np.sort(first), first)  # canonical: ids by first occurrence
     idx = np.random.default_rng(1).choice(len(X), 64, replace=False)
     assert oracle.terminal_violations(r["coords"], c.eps, lab, idx) == 0
+
+
+def test_pack_unpack_roundtrip_multi_rank_layout():
+    """The all-gather plumbing kernels: packing 3 rank ranges of D^{t+1} and unpacking the
+    concatenated (ranks*d, cnt) buffer reproduces the next state exactly (bitwise, ragged tail)."""
+    import torch
+    from paper_conf_edbt_jorgensena23_b200 import distributed as DR
+    X = datagen.blobs(1001, 3, 4, seed=3)
+    ref = E.Context(len(X), 3, 0.07)
+    ref.load(X)
+    it_ref, ok_ref, lab_ref = DR.run(ref)
+
+    class FakeComm:  # 3 "ranks" emulated in one process: every range is updated and exchanged
+        world, cnt = 3, (1001 + 2) // 3
+
+        def __init__(self):
+            self.lo, self.hi = 0, 1001
+
+        def reduce_min(self, v):
+            return v
+
+        def exchange(self, ctx):
+            parts = [torch.empty((3, self.cnt), device="cuda") for _ in range(3)]
+            for r in range(3):
+                ctx.pack_into(r * self.cnt, self.cnt, parts[r])
+            g = torch.cat(parts, 0)
+            ctx.unpack_from(g.view(3, -1, self.cnt), 3, self.cnt)
+
+    ctx = E.Context(len(X), 3, 0.07)
+    ctx.load(X)
+    it, ok, lab = DR.run(ctx, FakeComm())
+    assert ok and ok_ref and it == it_ref
+    assert np.array_equal(lab, lab_ref)
+    assert np.array_equal(ctx.coords(), ref.coords())
+
+
+def test_nccl_single_rank_driver():
+    """torch.distributed NCCL process group of size 1 through TorchComm equals the local run."""
+    import torch
+    import torch.distributed as dist
+    from paper_conf_edbt_jorgensena23_b200 import distributed as DR
+    X = datagen.blobs(3000, 4, 5, seed=1)
+    ref = E.cluster(X, 0.07)
+    os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+    os.environ.setdefault("MASTER_PORT", "29533")
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    try:
+        s = torch.cuda.Stream()
+        torch.cuda.set_stream(s)
+        ctx = E.Context(len(X), 4, 0.07, device=0, stream=s.cuda_stream)
+        ctx.load(X)
+        it, ok, lab = DR.run(ctx, DR.TorchComm(len(X), 4, torch.device("cuda", 0)))
+        assert ok and it == ref["iters"] and np.array_equal(lab, ref["labels"])
+    finally:
+        dist.destroy_process_group()
+        torch.cuda.set_stream(torch.cuda.default_stream())
