@@ -127,6 +127,12 @@ const char *eggsync_last_error(void);
 /* Library version string. */
 const char *eggsync_version(void);
 
+/* The library keeps the most recently released device workspace of each
+ * device (and its pinned flag buffer) cached for reuse by the next call that
+ * fits in it, so repeated calls do not pay cudaMalloc/cudaFree.  This frees
+ * the cache.  Not to be called concurrently with other library calls. */
+void eggsync_release_cache(void);
+
 /* ------------------------------------------------------------------------
  * Context (phase) API -- device-resident state for the multi-GPU driver and
  * for device-timed benchmarking.  Every pointer below is DEVICE memory on

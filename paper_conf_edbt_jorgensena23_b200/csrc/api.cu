@@ -7,7 +7,9 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstring>
+#include <mutex>
 #include <string>
+#include <vector>
 
 #include "common.cuh"
 
@@ -67,7 +69,64 @@ bool make_consts(int64_t n, int d, float eps, Consts* c, std::string* why) {
   return true;
 }
 
-// ------------------------------------------------------------------ workspace
+// ------------------------------------------------------------------ workspace cache
+// One released workspace arena (+ its pinned flag mirror) is kept per device and
+// reused by the next call that fits in it -- a caching allocator, so repeated
+// eggsync_cluster() calls do not pay cudaMalloc/cudaFree (eggsync_release_cache()).
+struct CachedArena {
+  int device;
+  char* p;
+  size_t bytes;
+  int32_t* hflags;
+};
+static std::mutex g_cache_mu;
+static std::vector<CachedArena> g_cache;
+
+static bool cache_take(int device, size_t need, char** p, size_t* bytes, int32_t** hflags) {
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  for (size_t k = 0; k < g_cache.size(); ++k) {
+    if (g_cache[k].device == device && g_cache[k].bytes >= need) {
+      *p = g_cache[k].p;
+      *bytes = g_cache[k].bytes;
+      *hflags = g_cache[k].hflags;
+      g_cache.erase(g_cache.begin() + k);
+      return true;
+    }
+  }
+  return false;
+}
+
+static void cache_give(int device, char* p, size_t bytes, int32_t* hflags) {
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  for (size_t k = 0; k < g_cache.size(); ++k) {
+    if (g_cache[k].device == device) {
+      if (g_cache[k].bytes >= bytes) {  // keep the larger one
+        cudaFree(p);
+        cudaFreeHost(hflags);
+        return;
+      }
+      cudaFree(g_cache[k].p);
+      cudaFreeHost(g_cache[k].hflags);
+      g_cache.erase(g_cache.begin() + k);
+      break;
+    }
+  }
+  g_cache.push_back({device, p, bytes, hflags});
+}
+
+static void cache_clear() {
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  int prev = -1;
+  cudaGetDevice(&prev);
+  for (auto& c : g_cache) {
+    cudaSetDevice(c.device);
+    cudaFree(c.p);
+    cudaFreeHost(c.hflags);
+  }
+  g_cache.clear();
+  if (prev >= 0) cudaSetDevice(prev);
+}
+
 int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
   std::string why;
   if (!make_consts(n_, d_, eps, &k, &why)) {
@@ -129,11 +188,23 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
   size_t total = 0;
   for (auto& it : items) total += (it.bytes + 255) & ~size_t(255);
   char* base = nullptr;
-  cudaError_t e = cudaMalloc((void**)&base, total);
-  if (e != cudaSuccess) {
-    set_error("cudaMalloc(%zu bytes) failed: %s", total, cudaGetErrorString(e));
-    cudaGetLastError();
-    return e == cudaErrorMemoryAllocation ? EGGSYNC_ENOMEM : EGGSYNC_ECUDA;
+  EGG_CUDA(cudaGetDevice(&cur_device));
+  size_t got = 0;
+  if (cache_take(cur_device, total, &base, &got, &h_flags)) {
+    total = got;
+  } else {
+    cudaError_t e = cudaMalloc((void**)&base, total);
+    if (e != cudaSuccess) {
+      set_error("cudaMalloc(%zu bytes) failed: %s", total, cudaGetErrorString(e));
+      cudaGetLastError();
+      return e == cudaErrorMemoryAllocation ? EGGSYNC_ENOMEM : EGGSYNC_ECUDA;
+    }
+    e = cudaMallocHost((void**)&h_flags, 16 * sizeof(int32_t));
+    if (e != cudaSuccess) {
+      cudaFree(base);
+      set_error("cudaMallocHost failed: %s", cudaGetErrorString(e));
+      return EGGSYNC_ENOMEM;
+    }
   }
   arena = base;
   size_t off = 0;
@@ -142,7 +213,6 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
     off += (it.bytes + 255) & ~size_t(255);
   }
   bytes = (int64_t)total;
-  EGG_CUDA(cudaMallocHost((void**)&h_flags, 16 * sizeof(int32_t)));
   if (st) {
     stream = st;
     own_stream = false;
@@ -157,9 +227,11 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
 }
 
 void Workspace::release() {
-  if (arena) cudaFree(arena);
+  if (arena) {
+    if (stream) cudaStreamSynchronize(stream);  // no pending work may touch a cached arena
+    cache_give(cur_device, arena, (size_t)bytes, h_flags);
+  }
   arena = nullptr;
-  if (h_flags) cudaFreeHost(h_flags);
   h_flags = nullptr;
   if (own_stream && stream) cudaStreamDestroy(stream);
   stream = nullptr;
@@ -357,6 +429,8 @@ extern "C" {
 
 const char* eggsync_last_error(void) { return g_err.c_str(); }
 const char* eggsync_version(void) { return "eggsync-b200 0.1 (sm_100a)"; }
+
+void eggsync_release_cache(void) { cache_clear(); }
 
 void eggsync_default_opts(eggsync_opts* o) {
   if (!o) return;

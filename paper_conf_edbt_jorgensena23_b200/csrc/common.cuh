@@ -185,6 +185,7 @@ struct Workspace {
   bool second_checked = false;
   int64_t bytes = 0;
   char* arena = nullptr;  // one device allocation carved into the arrays above
+  int cur_device = 0;     // device the arena lives on
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   int device = 0;

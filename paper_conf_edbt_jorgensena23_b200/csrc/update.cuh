@@ -37,10 +37,19 @@ namespace egg {
 #define EGG_UPD_BUCKET_SPARSE 256  // cells mostly singletons (early iterations)
 #define EGG_UPD_BUCKET_DENSE 64    // dense cells: box pruning pays
 #endif
+#ifndef EGG_UNCOND_ACC
+#define EGG_UNCOND_ACC 1
+#endif
+#ifndef EGG_UNROLL_G
+#define EGG_UNROLL_G 1
+#endif
 #ifndef EGG_UPD_MINB
 #define EGG_UPD_MINB 1
 #endif
-constexpr int kP = 2;                        // points per lane
+#ifndef EGG_PPL
+#define EGG_PPL 2
+#endif
+constexpr int kP = EGG_PPL;                  // points per lane
 // a subtree of <= a.bucket cells is processed cell by cell (chosen per launch, run_update)
 
 template <int D>
@@ -258,6 +267,9 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
     cb[4 * q + 2] = v.z;
     cb[4 * q + 3] = v.w;
   }
+#if EGG_UNROLL_G
+#pragma unroll 2
+#endif
   for (int g = 0; g < cntc; ++g, sg += SF) {
     bool in[kP], pa[kP];
     bool any_pa = false, any_in = false;
@@ -291,11 +303,28 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
         wc.acc += __popc(__ballot_sync(FULLMASK, in[k]));
       }
     }
+#if EGG_UNCOND_ACC
+    // masked accumulate without a vote/branch (>90% of staged cells are inside for some
+    // point); the summary loads are issued before the (rare) partial-cell branch
+    float sb[KB];
+#pragma unroll
+    for (int q = 0; q < KB / 4; ++q) {
+      const float4 v = reinterpret_cast<const float4*>(sg + KA)[q];
+      sb[4 * q] = v.x;
+      sb[4 * q + 1] = v.y;
+      sb[4 * q + 2] = v.z;
+      sb[4 * q + 3] = v.w;
+    }
+    const int cg = __float_as_int(sg[KA + KB]);
+#endif
     if (__any_sync(FULLMASK, any_pa)) {
 #pragma unroll
       for (int k = 0; k < kP; ++k)
         if (__any_sync(FULLMASK, pa[k])) scan_cell<D, CNT>(a, L, k, pa[k], first + g, sg, mst, lane, wc);
     }
+#if EGG_UNCOND_ACC
+    {
+#else
     if (__any_sync(FULLMASK, any_in)) {
       float sb[KB];
 #pragma unroll
@@ -307,6 +336,7 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
         sb[4 * q + 3] = v.w;
       }
       const int cg = __float_as_int(sg[KA + KB]);
+#endif
 #pragma unroll
       for (int k = 0; k < kP; ++k) {
         const float f = in[k] ? 1.f : 0.f;

@@ -26,6 +26,7 @@ SYMBOLS = [
     "eggsync_ctx_flags", "eggsync_ctx_cur_coords", "eggsync_ctx_next_coords", "eggsync_ctx_pack",
     "eggsync_ctx_unpack", "eggsync_ctx_advance", "eggsync_ctx_labels", "eggsync_ctx_coords",
     "eggsync_ctx_run", "eggsync_ctx_stream", "eggsync_ctx_work", "eggsync_ctx_launches",
+    "eggsync_release_cache",
 ]
 
 
@@ -91,6 +92,7 @@ def lib():
             "eggsync_ctx_stream": ([vp], vp),
             "eggsync_ctx_work": ([vp, i32, vp], ctypes.c_int),
             "eggsync_ctx_launches": ([vp], ctypes.c_int64),
+            "eggsync_release_cache": ([], None),
         }
         for name, (args, res) in sig.items():
             fn = getattr(L, name)
@@ -98,6 +100,11 @@ def lib():
             fn.restype = res
         _lib = L
     return _lib
+
+
+def release_cache() -> None:
+    """Free the library's cached device workspaces."""
+    lib().eggsync_release_cache()
 
 
 def last_error() -> str:
