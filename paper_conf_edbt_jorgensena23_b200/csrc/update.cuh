@@ -46,10 +46,15 @@ namespace egg {
 #ifndef EGG_UPD_MINB
 #define EGG_UPD_MINB 1
 #endif
-#ifndef EGG_PPL
-#define EGG_PPL 2
+// points per lane: 2 while the per-point state fits the register file, else 1
+template <int D>
+struct PPL {
+#ifdef EGG_PPL
+  static constexpr int v = EGG_PPL;
+#else
+  static constexpr int v = D <= 12 ? 2 : 1;
 #endif
-constexpr int kP = EGG_PPL;                  // points per lane
+};
 // a subtree of <= a.bucket cells is processed cell by cell (chosen per launch, run_update)
 
 template <int D>
@@ -110,6 +115,7 @@ __device__ __forceinline__ int popc64(unsigned long long m) { return __popcll(m)
 // Shared-memory layout of one warp (floats unless noted).
 template <int D>
 struct WarpSmem {
+  static constexpr int kP = PPL<D>::v;
   static constexpr int SF = Stage<D>::kFloats;
   static constexpr int OV = ceil4(D + 4);  // o[D], Bw, pad
   static constexpr int kStageFloats = 32 * SF;
@@ -121,6 +127,7 @@ struct WarpSmem {
 
 template <int D>
 struct Lane {
+  static constexpr int kP = PPL<D>::v;
   float q[kP][D];  // p - o (shifted point)
   float pp[kP];    // |q|^2
   float S[kP][D], C[kP][D];  // fp32 chunk accumulators
@@ -219,6 +226,7 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
                                             unsigned long long pm, float* __restrict__ st,
                                             const float* __restrict__ ov, double* __restrict__ mst,
                                             int lane, WorkCnt& wc) {
+  constexpr int kP = PPL<D>::v;
   constexpr int SF = Stage<D>::kFloats, KA = Stage<D>::kA, KB = Stage<D>::kB;
   constexpr int R = CellRec<D>::kFloats;
   __syncwarp();
@@ -267,10 +275,22 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
     cb[4 * q + 2] = v.z;
     cb[4 * q + 3] = v.w;
   }
-#if EGG_UNROLL_G
-#pragma unroll 2
-#endif
+  constexpr int kUnrollG = (EGG_UNROLL_G && D <= 12) ? 2 : 1;
+  constexpr bool kPrefetch = D <= 16;  // registers: high d reloads the A part in place
+#pragma unroll(kUnrollG)
   for (int g = 0; g < cntc; ++g, sg += SF) {
+    if constexpr (!kPrefetch) {
+      if (g > 0) {
+#pragma unroll
+        for (int q = 0; q < KA / 4; ++q) {
+          const float4 v = reinterpret_cast<const float4*>(sg)[q];
+          cb[4 * q] = v.x;
+          cb[4 * q + 1] = v.y;
+          cb[4 * q + 2] = v.z;
+          cb[4 * q + 3] = v.w;
+        }
+      }
+    }
     bool in[kP], pa[kP];
     bool any_pa = false, any_in = false;
 #pragma unroll
@@ -286,7 +306,7 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
       any_pa |= pa[k];
       any_in |= in[k];
     }
-    if (g + 1 < cntc) {  // software pipelining: next cell's A part
+    if (kPrefetch && g + 1 < cntc) {  // software pipelining: next cell's A part
 #pragma unroll
       for (int q = 0; q < KA / 4; ++q) {
         const float4 v = reinterpret_cast<const float4*>(sg + SF)[q];
@@ -303,30 +323,13 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
         wc.acc += __popc(__ballot_sync(FULLMASK, in[k]));
       }
     }
-#if EGG_UNCOND_ACC
-    // masked accumulate without a vote/branch (>90% of staged cells are inside for some
-    // point); the summary loads are issued before the (rare) partial-cell branch
+    // Low d: masked accumulate without a vote/branch (>90% of staged cells are inside
+    // for some point) with the summary loads issued before the (rare) partial-cell
+    // branch.  High d: load and accumulate only when some point is inside (registers).
+    constexpr bool kEarly = EGG_UNCOND_ACC && D <= 12;
     float sb[KB];
-#pragma unroll
-    for (int q = 0; q < KB / 4; ++q) {
-      const float4 v = reinterpret_cast<const float4*>(sg + KA)[q];
-      sb[4 * q] = v.x;
-      sb[4 * q + 1] = v.y;
-      sb[4 * q + 2] = v.z;
-      sb[4 * q + 3] = v.w;
-    }
-    const int cg = __float_as_int(sg[KA + KB]);
-#endif
-    if (__any_sync(FULLMASK, any_pa)) {
-#pragma unroll
-      for (int k = 0; k < kP; ++k)
-        if (__any_sync(FULLMASK, pa[k])) scan_cell<D, CNT>(a, L, k, pa[k], first + g, sg, mst, lane, wc);
-    }
-#if EGG_UNCOND_ACC
-    {
-#else
-    if (__any_sync(FULLMASK, any_in)) {
-      float sb[KB];
+    int cg = 0;
+    if constexpr (kEarly) {
 #pragma unroll
       for (int q = 0; q < KB / 4; ++q) {
         const float4 v = reinterpret_cast<const float4*>(sg + KA)[q];
@@ -335,8 +338,25 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
         sb[4 * q + 2] = v.z;
         sb[4 * q + 3] = v.w;
       }
-      const int cg = __float_as_int(sg[KA + KB]);
-#endif
+      cg = __float_as_int(sg[KA + KB]);
+    }
+    if (__any_sync(FULLMASK, any_pa)) {
+#pragma unroll
+      for (int k = 0; k < kP; ++k)
+        if (__any_sync(FULLMASK, pa[k])) scan_cell<D, CNT>(a, L, k, pa[k], first + g, sg, mst, lane, wc);
+    }
+    if (kEarly || __any_sync(FULLMASK, any_in)) {
+      if constexpr (!kEarly) {
+#pragma unroll
+        for (int q = 0; q < KB / 4; ++q) {
+          const float4 v = reinterpret_cast<const float4*>(sg + KA)[q];
+          sb[4 * q] = v.x;
+          sb[4 * q + 1] = v.y;
+          sb[4 * q + 2] = v.z;
+          sb[4 * q + 3] = v.w;
+        }
+        cg = __float_as_int(sg[KA + KB]);
+      }
 #pragma unroll
       for (int k = 0; k < kP; ++k) {
         const float f = in[k] ? 1.f : 0.f;
@@ -358,6 +378,7 @@ __device__ __forceinline__ void process_cells(const UpdArgs<D>& a, Lane<D>& L, i
                                               unsigned long long pm, float* __restrict__ st,
                                               const float* __restrict__ ov, double* __restrict__ mst,
                                               int lane, WorkCnt& wc) {
+  constexpr int kP = PPL<D>::v;
   for (int32_t r = 0; r < cntc; r += 32)
     stage_round<D, CNT>(a, L, first + r, min(32, cntc - r), pm, st, ov, mst, lane, wc);
 #pragma unroll
@@ -366,6 +387,7 @@ __device__ __forceinline__ void process_cells(const UpdArgs<D>& a, Lane<D>& L, i
 
 template <int D, bool CNT>
 __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(const UpdArgs<D> a) {
+  constexpr int kP = PPL<D>::v;
   using W = WarpSmem<D>;
   constexpr int BS = ceil4(2 * D);
   extern __shared__ __align__(16) float smem[];
@@ -463,32 +485,32 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(cons
     }
     const int node = ent.x;
     const float* __restrict__ bx = a.t_box + (int64_t)node * BS;
-    float lo[D], hi[D];
-#pragma unroll
-    for (int i = 0; i < D; ++i) {
-      lo[i] = bx[i] - ov[i];
-      hi[i] = bx[D + i] - ov[i];
-    }
     bool full[kP], part[kP];
     bool any_full = false;
+    float m0[kP], m1[kP], x0[kP], x1[kP];
+#pragma unroll
+    for (int k = 0; k < kP; ++k) m0[k] = m1[k] = x0[k] = x1[k] = 0.f;
+#pragma unroll
+    for (int i = 0; i < D; ++i) {  // box in the shifted frame, one dimension at a time
+      const float lo = bx[i] - ov[i], hi = bx[D + i] - ov[i];
+#pragma unroll
+      for (int k = 0; k < kP; ++k) {
+        const float dl = lo - L.q[k][i], dh = L.q[k][i] - hi;
+        const float mn = fmaxf(fmaxf(dl, dh), 0.f), mx = fmaxf(-dl, -dh);
+        if (i & 1) {
+          m1[k] = fmaf(mn, mn, m1[k]);
+          x1[k] = fmaf(mx, mx, x1[k]);
+        } else {
+          m0[k] = fmaf(mn, mn, m0[k]);
+          x0[k] = fmaf(mx, mx, x0[k]);
+        }
+      }
+    }
 #pragma unroll
     for (int k = 0; k < kP; ++k) {
       const bool act = (m >> (k * 32 + lane)) & 1ull;
-      float m0 = 0.f, m1 = 0.f, x0 = 0.f, x1 = 0.f;
-#pragma unroll
-      for (int i = 0; i < D; ++i) {
-        const float dl = lo[i] - L.q[k][i], dh = L.q[k][i] - hi[i];
-        const float mn = fmaxf(fmaxf(dl, dh), 0.f), mx = fmaxf(-dl, -dh);
-        if (i & 1) {
-          m1 = fmaf(mn, mn, m1);
-          x1 = fmaf(mx, mx, x1);
-        } else {
-          m0 = fmaf(mn, mn, m0);
-          x0 = fmaf(mx, mx, x0);
-        }
-      }
-      full[k] = act && (x0 + x1) <= lim_full;
-      part[k] = act && !full[k] && (m0 + m1) <= lim_out;
+      full[k] = act && (x0[k] + x1[k]) <= lim_full;
+      part[k] = act && !full[k] && (m0[k] + m1[k]) <= lim_out;
       any_full |= full[k];
     }
     if constexpr (CNT) {
@@ -607,7 +629,7 @@ int run_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   EGG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // all of the 228 KB unified L1/shared to shared memory: occupancy is shared-memory bound
   EGG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-  const int64_t pts_per_cta = 32 * kP * kWarpsPerCta;
+  const int64_t pts_per_cta = 32 * PPL<D>::v * kWarpsPerCta;
   const unsigned grid = (unsigned)((hi - lo + pts_per_cta - 1) / pts_per_cta);
   kern<<<grid, kWarpsPerCta * 32, smem, ws.stream>>>(a);
   ws.launches += 1;
