@@ -257,3 +257,29 @@ def test_nccl_single_rank_driver():
     finally:
         dist.destroy_process_group()
         torch.cuda.set_stream(torch.cuda.default_stream())
+
+
+# ------------------------------------------------- BASELINE configs C2 / C4
+def test_c2_full_oracle_parity():
+    """BASELINE config C2 (n=70,000, d=5, 10 clusters, eps=0.05) against the full O(T n^2 d)
+    oracle: identical labels, equal iteration count, coordinates within 1e-4 (~1 min of host CPU)."""
+    c = datagen.CONFIGS["C2"]
+    g, o = _cluster_compare(c.generate(0), c.eps)
+    assert g["iters"] == 7 and int(g["labels"].max()) + 1 == 24
+
+
+@pytest.mark.parametrize("d", [2, 5, 10, 15, 20])
+def test_c4_dimension_sweep_sampled(d):
+    """BASELINE config C4 (n=100,000, d=2..20, eps=0.05) at full size: the first update of
+    sampled points and their neighbour counts equal the oracle's per-point definition, and
+    the final clustering satisfies Theorem 4.7 for sampled points against all n."""
+    c = datagen.make_config(f"C4-d{d}")
+    X = c.generate(0)
+    g = E.step(X, c.eps, nbr=True)
+    idx = np.random.default_rng(d).choice(len(X), 256, replace=False)
+    Xs, ns = oracle.step_sample(X, c.eps, idx)
+    assert np.array_equal(g["nbr"][idx], ns)
+    assert np.abs(g["points"][idx].astype(np.float64) - Xs).max() <= 2e-6
+    r = E.cluster(X, c.eps, coords=True)
+    assert r["converged"]
+    assert oracle.terminal_violations(r["coords"], c.eps, r["labels"], idx[:64]) == 0
