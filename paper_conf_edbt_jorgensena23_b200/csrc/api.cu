@@ -6,6 +6,7 @@
 #include <chrono>
 #include <cmath>
 #include <cstdarg>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -52,12 +53,21 @@ bool make_consts(int64_t n, int d, float eps, Consts* c, std::string* why) {
   int bits = 0;
   while ((int64_t(1) << bits) < c->w) ++bits;
   c->bits = std::max(bits, 1);
-  c->keybits = d * c->bits;
-  c->nw = (c->keybits + 63) / 64;
-  if (c->nw > kMaxKeyWords) {
+  if (d * c->bits > 64 * kMaxKeyWords) {
     *why = "grid too fine: d*ceil(log2 w) > 512 key bits";
     return false;
   }
+  // Update units: each cell split into 2^(sub*d) sub-cells (F2).  In low d a cell holds
+  // many points and a ball boundary cuts through cells; finer units shrink the
+  // point-by-point boundary scan.  In high d cells are (near) singletons already.
+  // (measured on C2-C5, T1: finer is faster until units are ~single points)
+  static const int kSubByDim[21] = {0, 8, 8, 7, 6, 5, 5, 4, 3, 3, 2, 0, 0, 0, 0, 0, 0, 0, 0, 0, 0};
+  int sub = d <= 20 ? kSubByDim[d] : 0;
+  if (const char* s = getenv("EGGSYNC_SUBBITS")) sub = std::max(0, std::min(8, atoi(s)));
+  while (sub > 0 && d * (c->bits + sub) > 64 * kMaxKeyWords) --sub;
+  c->sub = sub;
+  c->keybits = d * (c->bits + sub);
+  c->nw = (c->keybits + 63) / 64;
   c->delta = c->e - c->e * std::sqrt(15.0 / 16.0) + c->e / 2.0 - std::sin(c->e / 2.0);  // L110
   c->ed = c->e + c->delta;
   c->ed2 = c->ed * c->ed;
@@ -184,6 +194,12 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
       {(void**)&nbr, sizeof(int32_t) * n},
       {(void**)&lab_final, sizeof(int32_t) * n},
       {(void**)&work, sizeof(unsigned long long) * 8},
+      {(void**)&co_of, sizeof(int32_t) * n},
+      {(void**)&co_start, sizeof(int32_t) * (cap + 1)},
+      {(void**)&co_cnt, sizeof(int32_t) * cap},
+      {(void**)&co_lo, sizeof(uint32_t) * d * cap},
+      {(void**)&co_hi, sizeof(uint32_t) * d * cap},
+      {(void**)&u2co, sizeof(int32_t) * cap},
   };
   size_t total = 0;
   for (auto& it : items) total += (it.bytes + 255) & ~size_t(255);
@@ -338,8 +354,8 @@ static int run_loop(Workspace& ws, int32_t max_iters, int32_t* iters_out, eggsyn
   for (;;) {
     EGG_TRY(iterate(ws, &synced, nullptr, nullptr, nullptr, stats));
     if (stats) {
-      if (t == 0) stats->n_cells_first = ws.n_cells;
-      stats->n_cells_last = ws.n_cells;
+      if (t == 0) stats->n_cells_first = ws.n_grid;
+      stats->n_cells_last = ws.n_grid;
     }
     if (synced) {
       if (stats) EGG_CUDA(cudaEventRecord(ws.ev[5], ws.stream));
@@ -590,7 +606,7 @@ int eggsync_ctx_build(eggsync_ctx* ctx, int32_t* n_cells_out) {
   ws.launches++;
   EGG_CUDA(cudaGetLastError());
   ws.second_checked = false;
-  if (n_cells_out) *n_cells_out = ws.n_cells;
+  if (n_cells_out) *n_cells_out = ws.n_grid;
   return EGGSYNC_OK;
 }
 

@@ -66,8 +66,9 @@ struct Consts {
   int64_t n;
   int d;
   int bits;    // bits per dimension of a cell coordinate: ceil(log2 w), >= 1
+  int sub;     // extra sub-cell bits per dimension (update units finer than the cells, F2)
   int nw;      // 64-bit words per Morton key
-  int keybits; // d * bits
+  int keybits; // d * (bits + sub)
   int64_t w;   // cells per dimension = ceil(1/c_w)          (Eq.4)
   double e, e2, cw, inv_cw, delta, ed, ed2;  // eps, eps^2, c_w (L252), 1/c_w, delta (L110), eps+delta
   float ef, e2f, edf, ed2f, rel;  // fp32 copies; rel = (4d+16) u relative safety margin
@@ -150,9 +151,25 @@ struct Workspace {
   // per point
   float* sn = nullptr;  // [d][n]
   float* cs = nullptr;
-  int32_t* cell_of = nullptr;  // [n]
+  int32_t* cell_of = nullptr;  // [n] update unit ("cell" below) of each sorted point
   int32_t* iscan = nullptr;    // [n] int scratch
-  // cells
+  // grid cells of width eps/(2 sqrt d) (L252): first term, second term, labels.
+  // Equal to the units when sub == 0; otherwise each cell is a run of units.
+  int32_t n_coarse = 0;
+  int32_t* co_of = nullptr;     // [n] cell of each sorted point
+  int32_t* co_start = nullptr;  // [cap+1]
+  int32_t* co_cnt = nullptr;    // [cap]
+  uint32_t* co_lo = nullptr;    // [d][cap] MBR (ordered bits)
+  uint32_t* co_hi = nullptr;
+  int32_t* u2co = nullptr;      // [cap] unit -> cell
+  // effective grid-cell arrays of the current build (alias the unit arrays when sub == 0)
+  int32_t n_grid = 0;
+  const int32_t* g_of = nullptr;
+  const int32_t* g_cnt = nullptr;
+  const uint32_t* g_lo = nullptr;
+  const uint32_t* g_hi = nullptr;
+  const int32_t* g_u2co = nullptr;  // nullptr: identity
+  // update units (summaries, hierarchy leaves)
   int32_t n_cells = 0;
   int32_t* cell_start = nullptr;  // [cap+1]
   uint64_t* c_fix = nullptr;      // [2d][cap]

@@ -39,8 +39,11 @@ __global__ void k_ingest(const float* __restrict__ io, int64_t n, int d, float* 
 }
 
 // --------------------------------------------------------------------- A1 keys
+// key of a point: Morton interleave of the fine coordinates f_i = c_i * 2^sub + s_i where
+// c_i is the cell coordinate and s_i the sub-cell (F2) inside it; the top D*cbits bits of
+// the code are the Morton code of the cell, so sorting groups cells, and sub-cells in them.
 template <int D>
-__global__ void k_keys(const float* __restrict__ xs, int64_t n, int bits, int nw, int64_t w,
+__global__ void k_keys(const float* __restrict__ xs, int64_t n, int cbits, int sub, int nw, int64_t w,
                        double inv_cw, uint64_t* __restrict__ keys) {
   int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (j >= n) return;
@@ -52,9 +55,15 @@ __global__ void k_keys(const float* __restrict__ xs, int64_t n, int bits, int nw
     int64_t ci = (int64_t)f;
     ci = ci > w - 1 ? w - 1 : ci;  // clamp x = 1.0 into the last cell (R2)
     ci = ci < 0 ? 0 : ci;
-    c[i] = (uint32_t)ci;
+    int64_t si = 0;
+    if (sub) {  // position inside the cell: t - ci is exact in fp64
+      si = (int64_t)floor(ldexp(t - (double)ci, sub));
+      si = si > (1 << sub) - 1 ? (1 << sub) - 1 : (si < 0 ? 0 : si);
+    }
+    c[i] = (uint32_t)((ci << sub) | si);
   }
   // Morton interleave, most significant bit-plane first: plane k holds bit (bits-1-k) of every c_i.
+  const int bits = cbits + sub;
   int widx = nw - 1;
   int filled = 64 * nw - D * bits;
   uint64_t acc = 0;
@@ -132,6 +141,72 @@ __global__ void k_cell_start(const int32_t* __restrict__ head, int32_t* __restri
     for (int w = 0; w < nw; ++w) c_key[(int64_t)w * cap + c] = keys[(int64_t)w * n + j];
   }
   if (j == n - 1) cell_start[c + 1] = (int32_t)n;
+}
+
+// Grid cells of width eps/(2 sqrt d) when update units are finer (sub > 0): two sorted
+// keys are in the same cell iff they agree above their lowest D*sub bits.
+__global__ void k_coarse_heads(const uint64_t* __restrict__ keys, int64_t n, int nw, int lowbits,
+                               int32_t* __restrict__ head) {
+  int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= n) return;
+  bool h = j == 0;
+  if (!h) {
+    for (int w = nw - 1; w >= 0; --w) {
+      uint64_t x = keys[(int64_t)w * n + j - 1], y = keys[(int64_t)w * n + j];
+      const int below = lowbits - 64 * w;  // sub-cell bits inside this word
+      if (below >= 64) break;
+      if (below > 0) {
+        x >>= below;
+        y >>= below;
+      }
+      if (x != y) {
+        h = true;
+        break;
+      }
+    }
+  }
+  head[j] = h;
+}
+
+__global__ void k_coarse_start(const int32_t* __restrict__ head, int32_t* __restrict__ co_of, int64_t n,
+                               int32_t* __restrict__ co_start) {
+  int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (j >= n) return;
+  const int32_t c = co_of[j] - 1;
+  co_of[j] = c;
+  if (head[j]) co_start[c] = (int32_t)j;
+  if (j == n - 1) co_start[c + 1] = (int32_t)n;
+}
+
+template <int D>
+__global__ void k_coarse_init(int32_t ncc, int64_t cap, const int32_t* __restrict__ co_start,
+                              int32_t* __restrict__ co_cnt, uint32_t* __restrict__ co_lo,
+                              uint32_t* __restrict__ co_hi) {
+  const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= ncc) return;
+  co_cnt[c] = co_start[c + 1] - co_start[c];
+#pragma unroll
+  for (int i = 0; i < D; ++i) {
+    co_lo[(int64_t)i * cap + c] = 0xffffffffu;
+    co_hi[(int64_t)i * cap + c] = 0u;
+  }
+}
+
+// unit -> cell map and cell MBR = union of its units' MBRs (order-independent atomics)
+template <int D>
+__global__ void k_coarse_mbr(int32_t nc, int64_t cap, const int32_t* __restrict__ cell_start,
+                             const int32_t* __restrict__ co_of, const uint32_t* __restrict__ c_lo,
+                             const uint32_t* __restrict__ c_hi, int32_t* __restrict__ u2co,
+                             uint32_t* __restrict__ co_lo, uint32_t* __restrict__ co_hi) {
+  const int64_t u = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (u >= nc) return;
+  const int32_t c = co_of[cell_start[u]];
+  u2co[u] = c;
+#pragma unroll
+  for (int i = 0; i < D; ++i) {
+    atomicMin(&co_lo[(int64_t)i * cap + c], c_lo[(int64_t)i * cap + u]);
+    atomicMax(&co_hi[(int64_t)i * cap + c], c_hi[(int64_t)i * cap + u]);
+  }
 }
 
 // -------------------------------------------------------------- A4 summaries
@@ -448,7 +523,7 @@ static int build_d(Workspace& ws) {
   cudaStream_t st = ws.stream;
   const int T = 256;
   // A1 keys of D^t in its current (previous sorted) order
-  k_keys<D><<<blocks_for(n, T), T, 0, st>>>(ws.xs[ws.xcur], n, K.bits, K.nw, K.w, K.inv_cw, ws.keys);
+  k_keys<D><<<blocks_for(n, T), T, 0, st>>>(ws.xs[ws.xcur], n, K.bits, K.sub, K.nw, K.w, K.inv_cw, ws.keys);
   EGG_LAUNCH_CHECK();
   EGG_CUDA(cudaMemsetAsync(ws.flags + 2, 0, sizeof(int32_t), st));
   if (n > 1) {
@@ -493,6 +568,16 @@ static int build_d(Workspace& ws) {
                                                ws.c_key);
   EGG_LAUNCH_CHECK();
   EGG_CUDA(cudaMemcpyAsync(ws.h_flags + 6, ws.cell_of + (n - 1), sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+  if (K.sub > 0) {  // grid cells above the update units
+    k_coarse_heads<<<blocks_for(n, T), T, 0, st>>>(ws.keys, n, K.nw, D * K.sub, ws.iscan);
+    EGG_LAUNCH_CHECK();
+    size_t bytes = ws.cub_bytes;
+    EGG_CUDA(cub::DeviceScan::InclusiveSum(ws.cub_tmp, bytes, ws.iscan, ws.co_of, (int)n, st));
+    ws.launches += 2;
+    k_coarse_start<<<blocks_for(n, T), T, 0, st>>>(ws.iscan, ws.co_of, n, ws.co_start);
+    EGG_LAUNCH_CHECK();
+    EGG_CUDA(cudaMemcpyAsync(ws.h_flags + 7, ws.co_of + (n - 1), sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+  }
   // A4 summaries
   if (n > 32) {
     k_init_span<D><<<blocks_for((n - 1) / 32, T), T, 0, st>>>(ws.cell_of, n, cap, ws.c_fix, ws.c_lo, ws.c_hi,
@@ -508,6 +593,27 @@ static int build_d(Workspace& ws) {
   k_cell_finalize<D><<<blocks_for(nc, T), T, 0, st>>>(nc, cap, ws.cell_start, ws.c_fix, ws.c_lo, ws.c_hi,
                                                       ws.c_cnt, ws.c_rec);
   EGG_LAUNCH_CHECK();
+  if (K.sub > 0) {
+    ws.n_grid = ws.h_flags[7] + 1;
+    k_coarse_init<D><<<blocks_for(ws.n_grid, T), T, 0, st>>>(ws.n_grid, cap, ws.co_start, ws.co_cnt, ws.co_lo,
+                                                            ws.co_hi);
+    EGG_LAUNCH_CHECK();
+    k_coarse_mbr<D><<<blocks_for(nc, T), T, 0, st>>>(nc, cap, ws.cell_start, ws.co_of, ws.c_lo, ws.c_hi, ws.u2co,
+                                                     ws.co_lo, ws.co_hi);
+    EGG_LAUNCH_CHECK();
+    ws.g_of = ws.co_of;
+    ws.g_cnt = ws.co_cnt;
+    ws.g_lo = ws.co_lo;
+    ws.g_hi = ws.co_hi;
+    ws.g_u2co = ws.u2co;
+  } else {  // units are the grid cells
+    ws.n_grid = nc;
+    ws.g_of = ws.cell_of;
+    ws.g_cnt = ws.c_cnt;
+    ws.g_lo = ws.c_lo;
+    ws.g_hi = ws.c_hi;
+    ws.g_u2co = nullptr;
+  }
   // A5 hierarchy
   if (nc > 1) {
     k_tree_build<<<blocks_for(nc - 1, T), T, 0, st>>>(ws.c_key, cap, K.nw, nc, ws.t_meta, ws.t_parent,
@@ -528,11 +634,11 @@ int stage_build(Workspace& ws) { EGG_DISPATCH(ws.d, build_d, ws); }
 
 int stage_labels(Workspace& ws, int32_t* labels_dev) {
   const int64_t n = ws.n;
-  const int32_t nc = ws.n_cells;
+  const int32_t nc = ws.n_grid;  // labels are grid cells (gatherCluster, L256)
   cudaStream_t st = ws.stream;
   const int T = 256;
   EGG_CUDA(cudaMemsetAsync(ws.c_minorig, 0xff, (size_t)nc * sizeof(uint32_t), st));
-  k_lab_min<<<blocks_for(n, T), T, 0, st>>>(ws.cell_of, ws.orig[ws.ocur], n, ws.c_minorig);
+  k_lab_min<<<blocks_for(n, T), T, 0, st>>>(ws.g_of, ws.orig[ws.ocur], n, ws.c_minorig);
   EGG_LAUNCH_CHECK();
   EGG_CUDA(cudaMemsetAsync(ws.i_lab, 0, (size_t)n * sizeof(int32_t), st));
   k_lab_flag<<<blocks_for(nc, T), T, 0, st>>>(ws.c_minorig, nc, ws.i_lab);
@@ -540,7 +646,7 @@ int stage_labels(Workspace& ws, int32_t* labels_dev) {
   size_t bytes = ws.cub_bytes;
   EGG_CUDA(cub::DeviceScan::ExclusiveSum(ws.cub_tmp, bytes, ws.i_lab, ws.iscan, (int)n, st));
   ws.launches += 2;
-  k_lab_write<<<blocks_for(n, T), T, 0, st>>>(ws.cell_of, ws.orig[ws.ocur], ws.c_minorig, ws.iscan, n, labels_dev);
+  k_lab_write<<<blocks_for(n, T), T, 0, st>>>(ws.g_of, ws.orig[ws.ocur], ws.c_minorig, ws.iscan, n, labels_dev);
   EGG_LAUNCH_CHECK();
   return EGGSYNC_OK;
 }

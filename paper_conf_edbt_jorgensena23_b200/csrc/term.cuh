@@ -15,10 +15,13 @@ namespace egg {
 template <int D>
 struct TermArgs {
   const float* __restrict__ xs;
-  const int32_t* __restrict__ cell_of;
-  const int32_t* __restrict__ cell_start;
-  const uint32_t* __restrict__ c_lo;
+  const int32_t* __restrict__ g_of;    // grid cell of each sorted point
+  const int32_t* __restrict__ u2co;    // unit -> grid cell (nullptr: identity)
+  const int32_t* __restrict__ cell_start;  // unit point ranges
+  const uint32_t* __restrict__ c_lo;   // unit MBR (candidate pruning)
   const uint32_t* __restrict__ c_hi;
+  const uint32_t* __restrict__ g_lo;   // grid cell MBR = MBR(N_{eps/2}(q)) under the first term
+  const uint32_t* __restrict__ g_hi;
   const int4* __restrict__ t_meta;
   const float* __restrict__ t_box;
   int64_t n, cap, lo, hi;
@@ -56,7 +59,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_second(const TermArgs<D> 
   float p[D];
 #pragma unroll
   for (int i = 0; i < D; ++i) p[i] = valid ? a.xs[(int64_t)i * a.n + j] : 0.f;
-  const int32_t own = valid ? a.cell_of[j] : -1;
+  const int32_t own = valid ? a.g_of[j] : -1;
   const float lim_ed = a.ed2f * (1.f + a.rel);
   const float e_in = a.e2f * (1.f - a.rel), e_out = a.e2f * (1.f + a.rel);
   const float ed_in = a.ed2f * (1.f - a.rel);
@@ -105,17 +108,26 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_second(const TermArgs<D> 
     }
     const bool pact = (pm >> lane) & 1u;
     for (int32_t c = first; c <= last; ++c) {
+      const int32_t gc = a.u2co ? a.u2co[c] : c;
+      // prune the unit by its own MBR (no point of it within eps + delta)
+      float umin = 0.f;
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        const float l = ordf(a.c_lo[(int64_t)i * a.cap + c]), h = ordf(a.c_hi[(int64_t)i * a.cap + c]);
+        const float mn = fmaxf(fmaxf(l - p[i], p[i] - h), 0.f);
+        umin = fmaf(mn, mn, umin);
+      }
       float lo[D], hi[D];
       float mind = 0.f;
 #pragma unroll
       for (int i = 0; i < D; ++i) {
-        lo[i] = ordf(a.c_lo[(int64_t)i * a.cap + c]);
-        hi[i] = ordf(a.c_hi[(int64_t)i * a.cap + c]);
+        lo[i] = ordf(a.g_lo[(int64_t)i * a.cap + gc]);
+        hi[i] = ordf(a.g_hi[(int64_t)i * a.cap + gc]);
         const float mn = fmaxf(fmaxf(lo[i] - p[i], p[i] - hi[i]), 0.f);
         mind = fmaf(mn, mn, mind);
       }
       // condition on q's MBR: dist(MBR(cell(q)), p) <= eps (L108), decided exactly near the margin
-      bool cand = pact && c != own && mind <= e_out;
+      bool cand = pact && gc != own && umin <= lim_ed && mind <= e_out;
       const bool amb = cand && mind > e_in;
       if (__any_sync(FULLMASK, amb)) {
         if (amb) cand = exact_mindist2<D>(lo, hi, p) <= a.e2d;
@@ -154,10 +166,13 @@ int run_second_term(Workspace& ws, int64_t lo, int64_t hi) {
   if (hi <= lo) return EGGSYNC_OK;
   TermArgs<D> a;
   a.xs = ws.xs[ws.xcur];
-  a.cell_of = ws.cell_of;
+  a.g_of = ws.g_of;
+  a.u2co = ws.g_u2co;
   a.cell_start = ws.cell_start;
   a.c_lo = ws.c_lo;
   a.c_hi = ws.c_hi;
+  a.g_lo = ws.g_lo;
+  a.g_hi = ws.g_hi;
   a.t_meta = ws.t_meta;
   a.t_box = ws.t_box;
   a.n = ws.n;

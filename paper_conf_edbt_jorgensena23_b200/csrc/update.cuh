@@ -63,8 +63,8 @@ struct UpdArgs {
   float* __restrict__ xs_next;   // D^{t+1}, SoA [D][n], sorted
   const float* __restrict__ sn;  // sin(x), SoA [D][n]
   const float* __restrict__ cs;  // cos(x)
-  const int32_t* __restrict__ cell_of;
-  const int32_t* __restrict__ c_cnt;
+  const int32_t* __restrict__ g_of;   // grid cell of each sorted point (first term, L252)
+  const int32_t* __restrict__ g_cnt;  // grid cell counts
   const float* __restrict__ c_rec;  // [nc][CellRec<D>::kFloats]
   const uint32_t* __restrict__ c_lo;  // [D][cap] ordered bits
   const uint32_t* __restrict__ c_hi;
@@ -572,7 +572,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(cons
         const double xn = x + (cx * Sd - sx * Cd) * inv;  // Eq.5
         a.xs_next[(int64_t)i * a.n + L.j[k]] = fminf(fmaxf((float)xn, 0.f), 1.f);
       }
-      f1 = f1 && (L.N[k] == a.c_cnt[a.cell_of[L.j[k]]]);  // Alg 3 l.14-15 (L248)
+      f1 = f1 && (L.N[k] == a.g_cnt[a.g_of[L.j[k]]]);  // Alg 3 l.14-15 (L248)
       if (a.nbr) a.nbr[L.j[k]] = L.N[k];
     }
   }
@@ -599,8 +599,8 @@ int run_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   a.xs_next = ws.xs[ws.xcur ^ 1];
   a.sn = ws.sn;
   a.cs = ws.cs;
-  a.cell_of = ws.cell_of;
-  a.c_cnt = ws.c_cnt;
+  a.g_of = ws.g_of;
+  a.g_cnt = ws.g_cnt;
   a.c_rec = ws.c_rec;
   a.c_lo = ws.c_lo;
   a.c_hi = ws.c_hi;
