@@ -161,7 +161,7 @@ def run_ours(args):
     torch.cuda.set_stream(stream)
     Xd = torch.from_numpy(X).to(dev)
     ctx = E.Context(n, d, c.eps, device=local, stream=stream.cuda_stream)
-    comm = DR.TorchComm(n, d, dev) if world > 1 else DR.LocalComm(n)
+    comm = DR.TorchComm(n, d, dev, ctx=ctx) if world > 1 else DR.LocalComm(n)
     flush = torch.empty(256 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)
 
     class Hooks:
@@ -266,7 +266,7 @@ def run_ours(args):
         "data": "synthetic",
         "config": {"workload": workload_desc(c), "n": n, "d": d, "eps": c.eps, "iters": iters,
                    "clustering_s": ms / 1e3, "clusters": int(lab.max()) + 1,
-                   "parallelism": f"replicate+own+allgather x{world}" if world > 1 else "single GPU",
+                   "parallelism": f"replicate + block-interleaved ownership + NCCL all-gather x{world}" if world > 1 else "single GPU",
                    "l2": "flushed between steps (256 MiB write); inputs resident in HBM",
                    "update_share_of_step": upd_share, "update_ms_per_launch": upd_avg,
                    "launches_per_step": launches / args.steps, "work_counters": work},

@@ -210,6 +210,18 @@ int eggsync_ctx_work(eggsync_ctx *ctx, int32_t enable, int64_t *totals_out);
  * counted per pass). */
 int64_t eggsync_ctx_launches(eggsync_ctx *ctx);
 
+/* Block-interleaved ownership for load balance across ranks: the update works on
+ * blocks of B = 64 (d <= 12) or 32 consecutive sorted points; rank r of `ranks`
+ * owns the blocks b with b % ranks == r (dense and sparse regions are spread over
+ * all ranks).  update_owned updates the owned points (like eggsync_ctx_update);
+ * owned_count returns the per-rank exchange size cnt = ceil(nblocks/ranks)*B;
+ * pack_owned writes the owned part of D^{t+1} to buf ([d][cnt], device, zero
+ * padded); unpack_owned scatters a gathered [ranks][d][cnt] device buffer back. */
+int eggsync_ctx_update_owned(eggsync_ctx *ctx, int32_t rank, int32_t ranks);
+int64_t eggsync_ctx_owned_count(eggsync_ctx *ctx, int32_t ranks);
+int eggsync_ctx_pack_owned(eggsync_ctx *ctx, int32_t rank, int32_t ranks, float *buf);
+int eggsync_ctx_unpack_owned(eggsync_ctx *ctx, const float *gathered, int32_t ranks);
+
 #ifdef __cplusplus
 }
 #endif

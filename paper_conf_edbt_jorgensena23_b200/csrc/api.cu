@@ -291,6 +291,37 @@ __global__ void k_unpack(const float* __restrict__ g, int64_t n, int d, int32_t 
   if (pos < n) xs[(int64_t)i * n + pos] = g[t];
 }
 
+// Block-interleaved ownership: rank r of R owns the update blocks b (B points each) with
+// b % R == r; its send buffer is [d][cnt], cnt = ceil(nblocks / R) * B (zero padded).
+__global__ void k_pack_owned(const float* __restrict__ xs, int64_t n, int d, int64_t B, int32_t r, int32_t R,
+                             int64_t cnt, float* __restrict__ buf) {
+  int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= cnt * d) return;
+  const int i = (int)(t / cnt);
+  const int64_t k = t - (int64_t)i * cnt;
+  const int64_t pos = ((k / B) * R + r) * B + (k % B);
+  buf[t] = pos < n ? xs[(int64_t)i * n + pos] : 0.f;
+}
+__global__ void k_unpack_owned(const float* __restrict__ g, int64_t n, int d, int64_t B, int32_t R, int64_t cnt,
+                               float* __restrict__ xs) {
+  int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= (int64_t)R * d * cnt) return;
+  const int64_t per_rank = (int64_t)d * cnt;
+  const int32_t r = (int32_t)(t / per_rank);
+  const int64_t rem = t - r * per_rank;
+  const int i = (int)(rem / cnt);
+  const int64_t k = rem - (int64_t)i * cnt;
+  const int64_t pos = ((k / B) * R + r) * B + (k % B);
+  if (pos < n) xs[(int64_t)i * n + pos] = g[t];
+}
+
+static int64_t owned_block_points(const Workspace& ws) { return 32 * (ws.d <= 12 ? 2 : 1); }  // = 32*ppl_for(d)
+static int64_t owned_count(const Workspace& ws, int32_t R) {
+  const int64_t B = owned_block_points(ws);
+  const int64_t nb = (ws.n + B - 1) / B;
+  return (nb + R - 1) / R * B;
+}
+
 static int read_flags(Workspace& ws, int32_t* f1, int32_t* f2, int32_t* err) {
   EGG_CUDA(cudaMemcpyAsync(ws.h_flags, ws.flags, 4 * sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
   EGG_CUDA(cudaStreamSynchronize(ws.stream));
@@ -720,5 +751,47 @@ int eggsync_ctx_work(eggsync_ctx* ctx, int32_t enable, int64_t* totals_out) {
 }
 
 int64_t eggsync_ctx_launches(eggsync_ctx* ctx) { return ctx ? ctx->ws.launches : -1; }
+
+int eggsync_ctx_update_owned(eggsync_ctx* ctx, int32_t rank, int32_t ranks) {
+  if (!ctx || ranks < 1 || rank < 0 || rank >= ranks) return EGGSYNC_EINVAL;
+  if (!ctx->ws.built) {
+    set_error("eggsync_ctx_update_owned before eggsync_ctx_build");
+    return EGGSYNC_EINVAL;
+  }
+  ctx->ws.own_stride = ranks;
+  ctx->ws.own_offset = rank;
+  const int rc = stage_update(ctx->ws, 0, ctx->ws.n, nullptr);
+  ctx->ws.own_stride = 1;
+  ctx->ws.own_offset = 0;
+  return rc;
+}
+
+int64_t eggsync_ctx_owned_count(eggsync_ctx* ctx, int32_t ranks) {
+  if (!ctx || ranks < 1) return -1;
+  return owned_count(ctx->ws, ranks);
+}
+
+int eggsync_ctx_pack_owned(eggsync_ctx* ctx, int32_t rank, int32_t ranks, float* buf) {
+  if (!ctx || !buf || ranks < 1 || rank < 0 || rank >= ranks) return EGGSYNC_EINVAL;
+  Workspace& ws = ctx->ws;
+  const int64_t cnt = owned_count(ws, ranks), tot = cnt * ws.d;
+  k_pack_owned<<<(unsigned)((tot + 255) / 256), 256, 0, ws.stream>>>(ws.xs[ws.xcur ^ 1], ws.n, ws.d,
+                                                                      owned_block_points(ws), rank, ranks, cnt, buf);
+  ws.launches++;
+  EGG_CUDA(cudaGetLastError());
+  return EGGSYNC_OK;
+}
+
+int eggsync_ctx_unpack_owned(eggsync_ctx* ctx, const float* gathered, int32_t ranks) {
+  if (!ctx || !gathered || ranks < 1) return EGGSYNC_EINVAL;
+  Workspace& ws = ctx->ws;
+  const int64_t cnt = owned_count(ws, ranks), tot = (int64_t)ranks * ws.d * cnt;
+  k_unpack_owned<<<(unsigned)((tot + 255) / 256), 256, 0, ws.stream>>>(gathered, ws.n, ws.d, owned_block_points(ws),
+                                                                        ranks, cnt, ws.xs[ws.xcur ^ 1]);
+  ws.launches++;
+  EGG_CUDA(cudaGetLastError());
+  return EGGSYNC_OK;
+}
+
 
 }  // extern "C"

@@ -212,6 +212,7 @@ struct Workspace {
   unsigned long long* work = nullptr;  // [8] work counters of the instrumented update
   bool count_work = false;
   int64_t launches = 0;  // kernel launches issued on this workspace (CUB internals counted by pass)
+  int32_t own_stride = 1, own_offset = 0;  // block-interleaved ownership of the next update
 
   int alloc(int64_t n, int d, float eps, int device, cudaStream_t stream);
   void release();

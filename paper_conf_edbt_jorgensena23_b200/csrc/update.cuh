@@ -47,13 +47,16 @@ namespace egg {
 #define EGG_UPD_MINB 1
 #endif
 // points per lane: 2 while the per-point state fits the register file, else 1
+__host__ __device__ constexpr int ppl_for(int d) {
+#ifdef EGG_PPL
+  return EGG_PPL;
+#else
+  return d <= 12 ? 2 : 1;
+#endif
+}
 template <int D>
 struct PPL {
-#ifdef EGG_PPL
-  static constexpr int v = EGG_PPL;
-#else
-  static constexpr int v = D <= 12 ? 2 : 1;
-#endif
+  static constexpr int v = ppl_for(D);
 };
 // a subtree of <= a.bucket cells is processed cell by cell (chosen per launch, run_update)
 
@@ -74,6 +77,7 @@ struct UpdArgs {
   const int32_t* __restrict__ t_cnt;
   int64_t n, cap, lo, hi;
   int32_t nc, stack_len, bucket;
+  int32_t stride, offset;  // this launch owns the 32*kP-point blocks b = stride*w + offset
   float e, e2f, rel;
   double e2d;
   int32_t* flags;  // [0] first term AND, [3] error
@@ -399,7 +403,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(cons
   double* mst = reinterpret_cast<double*>(wbase + (size_t)(W::kStageFloats + W::OV) * 4);
   int4* stk = reinterpret_cast<int4*>(wbase + (size_t)(W::kStageFloats + W::OV) * 4 + (size_t)W::kMasterDoubles * 8);
 
-  const int64_t base = a.lo + ((int64_t)blockIdx.x * kWarpsPerCta + wid) * (32 * kP);
+  const int64_t base = a.lo + (((int64_t)blockIdx.x * kWarpsPerCta + wid) * a.stride + a.offset) * (32 * kP);
   Lane<D> L;
   unsigned long long amask = 0ull;
 #pragma unroll
@@ -629,8 +633,14 @@ int run_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   EGG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // all of the 228 KB unified L1/shared to shared memory: occupancy is shared-memory bound
   EGG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, 100));
-  const int64_t pts_per_cta = 32 * PPL<D>::v * kWarpsPerCta;
-  const unsigned grid = (unsigned)((hi - lo + pts_per_cta - 1) / pts_per_cta);
+  // block-interleaved ownership (multi-GPU load balance): blocks b with b % stride == offset
+  a.stride = ws.own_stride;
+  a.offset = ws.own_offset;
+  const int64_t B = 32 * PPL<D>::v;
+  const int64_t nblocks = (hi - lo + B - 1) / B;
+  const int64_t owned = nblocks > a.offset ? (nblocks - a.offset + a.stride - 1) / a.stride : 0;
+  if (owned == 0) return EGGSYNC_OK;
+  const unsigned grid = (unsigned)((owned + kWarpsPerCta - 1) / kWarpsPerCta);
   kern<<<grid, kWarpsPerCta * 32, smem, ws.stream>>>(a);
   ws.launches += 1;
   EGG_CUDA(cudaGetLastError());

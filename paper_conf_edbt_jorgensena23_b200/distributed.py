@@ -1,14 +1,17 @@
 """Algorithm 4 over the phase API, single- or multi-rank.
 
-Multi-GPU scheme ("replicate + own + all-gather"):
-every rank holds all n points and builds the identical structure (the build
-is deterministic: Morton keys, stable sort, integer summaries), updates only
-its contiguous range [lo, hi) of the sorted order (Eq.1 is a Jacobi update,
-L68, so ranges are independent given D^t), then the ranks exchange their
-updated ranges with one all-gather (NCCL over NVLink via torch.distributed)
-and AND-reduce the two criterion flags.  The result is bitwise identical to
-one GPU.  torch.distributed is plumbing only; all arithmetic is in the
-library's kernels.
+Multi-GPU scheme ("replicate + own + all-gather"): every rank
+holds all n points and builds the identical structure (the build is
+deterministic: Morton keys, stable sort, integer summaries), updates only the
+points it owns (Eq.1 is a Jacobi update, L68, so owned sets are independent
+given D^t), then the ranks exchange their updated points with one all-gather
+(NCCL over NVLink via torch.distributed) and AND-reduce the two criterion
+flags.  The result is bitwise identical to one GPU.
+
+Ownership is block-interleaved by default: the update's 64-point blocks of the
+sorted order are dealt round-robin to the ranks, so dense cluster cores and
+sparse noise are spread evenly (a contiguous split gives one rank the dense
+core).  torch.distributed is plumbing only; all arithmetic is in the library.
 """
 from __future__ import annotations
 
@@ -24,22 +27,38 @@ class LocalComm:
     def reduce_min(self, v: int) -> int:
         return v
 
+    def update(self, ctx) -> None:
+        ctx.update(self.lo, self.hi)
+
     def exchange(self, ctx) -> None:
         pass
 
 
 class TorchComm:
-    """Rank r owns sorted positions [r*cnt, min(n, (r+1)*cnt)), cnt = ceil(n / world)."""
+    """One rank of a torch.distributed group.
 
-    def __init__(self, n: int, d: int, device, group=None):
+    mode "interleaved": update blocks b with b % world == rank (load balance);
+    mode "contiguous" : rank r owns sorted positions [r*cnt, min(n, (r+1)*cnt)).
+    The second criterion term is split contiguously in both modes.
+    """
+
+    def __init__(self, n: int, d: int, device, group=None, mode: str = "interleaved", ctx=None):
         import torch
         import torch.distributed as dist
-        self.dist, self.group = dist, group
+        self.dist, self.group, self.mode = dist, group, mode
         self.world = dist.get_world_size(group)
         self.rank = dist.get_rank(group)
-        self.cnt = math.ceil(n / self.world)
-        self.lo = min(n, self.rank * self.cnt)
-        self.hi = min(n, self.lo + self.cnt)
+        span = math.ceil(n / self.world)
+        self.lo = min(n, self.rank * span)                  # contiguous share (second term)
+        self.hi = min(n, self.lo + span)
+        if mode == "interleaved":
+            if ctx is None:
+                raise ValueError("interleaved ownership needs the context (block size)")
+            self.cnt = ctx.owned_count(self.world)
+        elif mode == "contiguous":
+            self.cnt = span
+        else:
+            raise ValueError(mode)
         self.send = torch.empty((d, self.cnt), dtype=torch.float32, device=device)
         # concatenated layout (world*d, cnt) == stacked (world, d, cnt) in memory (gloo needs the former)
         self.recv = torch.empty((self.world * d, self.cnt), dtype=torch.float32, device=device)
@@ -50,10 +69,23 @@ class TorchComm:
         self.dist.all_reduce(self.flag, op=self.dist.ReduceOp.MIN, group=self.group)
         return int(self.flag.item())
 
+    def update(self, ctx) -> None:
+        if self.mode == "interleaved":
+            ctx.update_owned(self.rank, self.world)
+        else:
+            ctx.update(self.lo, self.hi)
+
     def exchange(self, ctx) -> None:
-        ctx.pack_into(self.lo, self.cnt, self.send)
+        if self.mode == "interleaved":
+            ctx.pack_owned_into(self.rank, self.world, self.send)
+        else:
+            ctx.pack_into(self.lo, self.cnt, self.send)
         self.dist.all_gather_into_tensor(self.recv, self.send, group=self.group)
-        ctx.unpack_from(self.recv.view(self.world, -1, self.cnt), self.world, self.cnt)
+        view = self.recv.view(self.world, -1, self.cnt)
+        if self.mode == "interleaved":
+            ctx.unpack_owned_from(view, self.world)
+        else:
+            ctx.unpack_from(view, self.world, self.cnt)
 
 
 def run(ctx, comm=None, max_iters: int = 10000, hooks=None):
@@ -70,7 +102,7 @@ def run(ctx, comm=None, max_iters: int = 10000, hooks=None):
         ctx.build()
         if hooks:
             hooks.before_update()
-        ctx.update(comm.lo, comm.hi)                      # Alg 3 on the owned range
+        comm.update(ctx)                                  # Alg 3 on the owned points
         if hooks:
             hooks.after_update()
         f1 = comm.reduce_min(ctx.flags()[0])              # first term (Alg 3 l.14-15)

@@ -26,7 +26,8 @@ SYMBOLS = [
     "eggsync_ctx_flags", "eggsync_ctx_cur_coords", "eggsync_ctx_next_coords", "eggsync_ctx_pack",
     "eggsync_ctx_unpack", "eggsync_ctx_advance", "eggsync_ctx_labels", "eggsync_ctx_coords",
     "eggsync_ctx_run", "eggsync_ctx_stream", "eggsync_ctx_work", "eggsync_ctx_launches",
-    "eggsync_release_cache",
+    "eggsync_release_cache", "eggsync_ctx_update_owned", "eggsync_ctx_owned_count", "eggsync_ctx_pack_owned",
+    "eggsync_ctx_unpack_owned",
 ]
 
 
@@ -93,6 +94,10 @@ def lib():
             "eggsync_ctx_work": ([vp, i32, vp], ctypes.c_int),
             "eggsync_ctx_launches": ([vp], ctypes.c_int64),
             "eggsync_release_cache": ([], None),
+            "eggsync_ctx_update_owned": ([vp, i32, i32], ctypes.c_int),
+            "eggsync_ctx_owned_count": ([vp, i32], ctypes.c_int64),
+            "eggsync_ctx_pack_owned": ([vp, i32, i32, vp], ctypes.c_int),
+            "eggsync_ctx_unpack_owned": ([vp, vp, i32], ctypes.c_int),
         }
         for name, (args, res) in sig.items():
             fn = getattr(L, name)
@@ -260,6 +265,19 @@ class Context:
     def unpack_from(self, tensor, ranks: int, cnt: int):
         """Gathered (ranks, d, cnt) CUDA tensor into the next-state buffer."""
         self.unpack(tensor.data_ptr(), ranks, cnt)
+
+    # block-interleaved ownership (multi-GPU load balance)
+    def update_owned(self, rank: int, ranks: int):
+        _check(lib().eggsync_ctx_update_owned(self.h, rank, ranks))
+
+    def owned_count(self, ranks: int) -> int:
+        return int(lib().eggsync_ctx_owned_count(self.h, ranks))
+
+    def pack_owned_into(self, rank: int, ranks: int, tensor):
+        _check(lib().eggsync_ctx_pack_owned(self.h, rank, ranks, ctypes.c_void_p(tensor.data_ptr())))
+
+    def unpack_owned_from(self, tensor, ranks: int):
+        _check(lib().eggsync_ctx_unpack_owned(self.h, ctypes.c_void_p(tensor.data_ptr()), ranks))
 
     def advance(self):
         _check(lib().eggsync_ctx_advance(self.h))

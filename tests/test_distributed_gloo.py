@@ -71,6 +71,38 @@ class OracleCtx:
     def flags(self):
         return self.f[0], (self.f[1] if self.checked else -1)
 
+    # block-interleaved ownership (same index map as the library, block size B)
+    B = 8
+
+    def owned_count(self, R):
+        nb = -(-self.n // self.B)
+        return -(-nb // R) * self.B
+
+    def _owned_pos(self, r, R, cnt):
+        k = np.arange(cnt)
+        return ((k // self.B) * R + r) * self.B + k % self.B
+
+    def update_owned(self, r, R):
+        pos = self._owned_pos(r, R, self.owned_count(R))
+        pos = pos[pos < self.n]
+        self.nxt[pos] = self.Xn[pos]
+        self.f[0] &= int(self.f1p[pos].all())
+
+    def pack_owned_into(self, r, R, t):
+        cnt = self.owned_count(R)
+        pos = self._owned_pos(r, R, cnt)
+        t.zero_()
+        ok = pos < self.n
+        t[:, np.nonzero(ok)[0]] = torch.from_numpy(self.nxt[pos[ok]].T.astype(np.float32))
+
+    def unpack_owned_from(self, t, R):
+        cnt = self.owned_count(R)
+        g = t.numpy().astype(np.float64)
+        for r in range(R):
+            pos = self._owned_pos(r, R, cnt)
+            ok = pos < self.n
+            self.nxt[pos[ok]] = g[r][:, ok].T
+
     def pack_into(self, lo, cnt, t):
         t.zero_()
         k = max(0, min(cnt, self.n - lo))
@@ -98,21 +130,22 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, X, eps, out):
+def _worker(rank, world, port, X, eps, out, mode):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
         ctx = OracleCtx(X.astype(np.float32), eps)
-        comm = DR.TorchComm(ctx.n, ctx.d, "cpu")
+        comm = DR.TorchComm(ctx.n, ctx.d, "cpu", mode=mode, ctx=ctx)
         it, ok, lab = DR.run(ctx, comm)
         out[rank] = (it, ok, lab.tolist(), ctx.X.tolist(), comm.lo, comm.hi)
     finally:
         dist.destroy_process_group()
 
 
+@pytest.mark.parametrize("mode", ["interleaved", "contiguous"])
 @pytest.mark.parametrize("n,d,k,eps,seed", [(60, 2, 3, 0.08, 0), (75, 3, 4, 0.12, 1)])
-def test_two_rank_run_equals_single_process(n, d, k, eps, seed):
+def test_two_rank_run_equals_single_process(n, d, k, eps, seed, mode):
     X = datagen.blobs(n, d, k, seed=seed)
     # exchange in fp32 (the library's state type): the single-process reference does the same
     ref = OracleCtx(X, eps)
@@ -120,7 +153,7 @@ def test_two_rank_run_equals_single_process(n, d, k, eps, seed):
     mgr = mp.Manager()
     out = mgr.dict()
     port = _free_port()
-    mp.spawn(_worker, args=(2, port, X, eps, out), nprocs=2, join=True)
+    mp.spawn(_worker, args=(2, port, X, eps, out, mode), nprocs=2, join=True)
     assert set(out.keys()) == {0, 1}
     (it0, ok0, lab0, X0, lo0, hi0), (it1, ok1, lab1, X1, lo1, hi1) = out[0], out[1]
     assert (lo0, hi0, lo1, hi1) == (0, (n + 1) // 2, (n + 1) // 2, n)

@@ -222,6 +222,9 @@ def test_pack_unpack_roundtrip_multi_rank_layout():
         def reduce_min(self, v):
             return v
 
+        def update(self, ctx):
+            ctx.update(self.lo, self.hi)
+
         def exchange(self, ctx):
             parts = [torch.empty((3, self.cnt), device="cuda") for _ in range(3)]
             for r in range(3):
@@ -235,6 +238,24 @@ def test_pack_unpack_roundtrip_multi_rank_layout():
     assert ok and ok_ref and it == it_ref
     assert np.array_equal(lab, lab_ref)
     assert np.array_equal(ctx.coords(), ref.coords())
+
+    class FakeOwned(FakeComm):  # block-interleaved ownership, 3 emulated ranks
+        def update(self, ctx):
+            for r in range(3):
+                ctx.update_owned(r, 3)
+
+        def exchange(self, ctx):
+            cnt = ctx.owned_count(3)
+            parts = [torch.empty((3, cnt), device="cuda") for _ in range(3)]
+            for r in range(3):
+                ctx.pack_owned_into(r, 3, parts[r])
+            ctx.unpack_owned_from(torch.cat(parts, 0).view(3, -1, cnt), 3)
+
+    ctx2 = E.Context(len(X), 3, 0.07)
+    ctx2.load(X)
+    it2, ok2, lab2 = DR.run(ctx2, FakeOwned())
+    assert ok2 and it2 == it_ref and np.array_equal(lab2, lab_ref)
+    assert np.array_equal(ctx2.coords(), ref.coords())
 
 
 def test_nccl_single_rank_driver():
@@ -252,7 +273,7 @@ def test_nccl_single_rank_driver():
         torch.cuda.set_stream(s)
         ctx = E.Context(len(X), 4, 0.07, device=0, stream=s.cuda_stream)
         ctx.load(X)
-        it, ok, lab = DR.run(ctx, DR.TorchComm(len(X), 4, torch.device("cuda", 0)))
+        it, ok, lab = DR.run(ctx, DR.TorchComm(len(X), 4, torch.device("cuda", 0), ctx=ctx))
         assert ok and it == ref["iters"] and np.array_equal(lab, ref["labels"])
     finally:
         dist.destroy_process_group()
