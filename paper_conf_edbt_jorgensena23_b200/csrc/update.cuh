@@ -123,10 +123,46 @@ struct WarpSmem {
   static constexpr int SF = Stage<D>::kFloats;
   static constexpr int OV = ceil4(D + 4);  // o[D], Bw, pad
   static constexpr int kStageFloats = 32 * SF;
+  static constexpr int kRawFloats = 2 * 32 * CellRec<D>::kFloats;  // TMA double buffer of cell records
   static constexpr int kMasterDoubles = kP * 2 * D * 32;
-  __host__ __device__ static size_t bytes(int stack_len) {
-    return (size_t)(kStageFloats + OV) * 4 + (size_t)kMasterDoubles * 8 + (size_t)stack_len * 16;
-  }
+  // [stage | ov | raw[2] floats][2 mbarriers][masters doubles][stack int4]
+  __host__ __device__ static constexpr size_t off_bar() { return (size_t)(kStageFloats + OV + kRawFloats) * 4; }
+  __host__ __device__ static constexpr size_t off_mst() { return off_bar() + 16; }
+  __host__ __device__ static constexpr size_t off_stk() { return off_mst() + (size_t)kMasterDoubles * 8; }
+  __host__ __device__ static size_t bytes(int stack_len) { return off_stk() + (size_t)stack_len * 16; }
+};
+
+// ---- TMA (cp.async.bulk) staging of cell records: global -> shared, mbarrier completion
+__device__ __forceinline__ unsigned smem_u32(const void* p) {
+  return static_cast<unsigned>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void tma_load_1d(void* dst, const void* src, unsigned bytes, uint64_t* bar) {
+  // order earlier generic-proxy accesses of dst before the async-proxy write
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, unsigned parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra WAIT_%=;\n}" ::"r"(
+          smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+
+// Per-warp TMA staging state (warp-uniform): two record buffers, their barriers and phases.
+struct TmaStage {
+  float* raw;      // raw[2][32 * CellRec<D>::kFloats]
+  uint64_t* bar;   // bar[2]
+  unsigned phase;  // bit b = parity of the next completion of buffer b
 };
 
 template <int D>
@@ -229,13 +265,13 @@ template <int D, bool CNT>
 __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int32_t first, int32_t cntc,
                                             unsigned long long pm, float* __restrict__ st,
                                             const float* __restrict__ ov, double* __restrict__ mst,
-                                            int lane, WorkCnt& wc) {
+                                            int lane, WorkCnt& wc, const float* __restrict__ raw) {
   constexpr int kP = PPL<D>::v;
   constexpr int SF = Stage<D>::kFloats, KA = Stage<D>::kA, KB = Stage<D>::kB;
   constexpr int R = CellRec<D>::kFloats;
   __syncwarp();
   if (lane < cntc) {
-    const float* __restrict__ r = a.c_rec + (int64_t)(first + lane) * R;
+    const float* __restrict__ r = raw + lane * R;  // record staged by the TMA bulk copy
     float* dst = st + lane * SF;
     const float Bw = ov[D];
     float cc = 0.f;
@@ -381,10 +417,25 @@ template <int D, bool CNT>
 __device__ __forceinline__ void process_cells(const UpdArgs<D>& a, Lane<D>& L, int32_t first, int32_t cntc,
                                               unsigned long long pm, float* __restrict__ st,
                                               const float* __restrict__ ov, double* __restrict__ mst,
-                                              int lane, WorkCnt& wc) {
+                                              int lane, WorkCnt& wc, TmaStage& tma) {
   constexpr int kP = PPL<D>::v;
-  for (int32_t r = 0; r < cntc; r += 32)
-    stage_round<D, CNT>(a, L, first + r, min(32, cntc - r), pm, st, ov, mst, lane, wc);
+  constexpr int R = CellRec<D>::kFloats;
+  const int nr = (cntc + 31) / 32;
+  // round r's 32 records are fetched with one bulk copy while round r-1 is processed
+  __syncwarp();
+  if (lane == 0) tma_load_1d(tma.raw, a.c_rec + (int64_t)first * R, (unsigned)min(32, cntc) * R * 4, tma.bar);
+  for (int r = 0; r < nr; ++r) {
+    const int b = r & 1;
+    if (r + 1 < nr && lane == 0) {
+      const int c1 = min(32, cntc - 32 * (r + 1));
+      tma_load_1d(tma.raw + (b ^ 1) * 32 * R, a.c_rec + (int64_t)(first + 32 * (r + 1)) * R, (unsigned)c1 * R * 4,
+                  tma.bar + (b ^ 1));
+    }
+    mbar_wait(tma.bar + b, (tma.phase >> b) & 1u);
+    tma.phase ^= 1u << b;
+    stage_round<D, CNT>(a, L, first + 32 * r, min(32, cntc - 32 * r), pm, st, ov, mst, lane, wc,
+                        tma.raw + b * 32 * R);
+  }
 #pragma unroll
   for (int k = 0; k < kP; ++k) flush(L, k, mst, lane);
 }
@@ -400,8 +451,12 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(cons
   char* wbase = reinterpret_cast<char*>(smem) + (size_t)wid * W::bytes(a.stack_len);
   float* st = reinterpret_cast<float*>(wbase);
   float* ov = st + W::kStageFloats;
-  double* mst = reinterpret_cast<double*>(wbase + (size_t)(W::kStageFloats + W::OV) * 4);
-  int4* stk = reinterpret_cast<int4*>(wbase + (size_t)(W::kStageFloats + W::OV) * 4 + (size_t)W::kMasterDoubles * 8);
+  TmaStage tma;
+  tma.raw = ov + W::OV;
+  tma.bar = reinterpret_cast<uint64_t*>(wbase + W::off_bar());
+  tma.phase = 0u;
+  double* mst = reinterpret_cast<double*>(wbase + W::off_mst());
+  int4* stk = reinterpret_cast<int4*>(wbase + W::off_stk());
 
   const int64_t base = a.lo + (((int64_t)blockIdx.x * kWarpsPerCta + wid) * a.stride + a.offset) * (32 * kP);
   Lane<D> L;
@@ -471,6 +526,11 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(cons
   const float lim_full = nfu * nfu * (1.f - (float)(2 * D + 8) * kU);
   if (lane == 0) ov[D] = Bw;
   for (int t = lane; t < W::kMasterDoubles; t += 32) mst[t] = 0.0;
+  if (lane == 0) {
+    mbar_init(tma.bar, 1);
+    mbar_init(tma.bar + 1, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
   __syncwarp();
 
   WorkCnt wc;
@@ -484,7 +544,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(cons
     __syncwarp();
     const unsigned long long m = (unsigned long long)(uint32_t)ent.y | ((unsigned long long)(uint32_t)ent.z << 32);
     if (ent.x & (int)kLeafBit) {
-      process_cells<D, CNT>(a, L, ent.x & 0x7fffffff, 1, m, st, ov, mst, lane, wc);
+      process_cells<D, CNT>(a, L, ent.x & 0x7fffffff, 1, m, st, ov, mst, lane, wc, tma);
       continue;
     }
     const int node = ent.x;
@@ -547,7 +607,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(cons
     if (pm == 0ull) continue;
     const int4 meta = a.t_meta[node];
     if (meta.y - meta.x + 1 <= a.bucket) {
-      process_cells<D, CNT>(a, L, meta.x, meta.y - meta.x + 1, pm, st, ov, mst, lane, wc);
+      process_cells<D, CNT>(a, L, meta.x, meta.y - meta.x + 1, pm, st, ov, mst, lane, wc, tma);
     } else {
       if (sp + 2 > a.stack_len) {  // cannot happen for depth <= key bits; guard anyway
         if (lane == 0) atomicExch(&a.flags[3], 1);
