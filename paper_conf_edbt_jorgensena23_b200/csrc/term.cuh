@@ -67,8 +67,10 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_second(const TermArgs<D> 
   int sp = 1;
   if (lane == 0) stk[0] = make_int2(a.nc > 1 ? 0 : (int)kLeafBit, (int)amask);
   __syncwarp();
+  int pops = 0;
   while (sp > 0) {
-    if (*(volatile int32_t*)&a.flags[1] == 0) break;  // someone already found a violation
+    // early exit once any warp found a violation (polled every 64 pops: an L2 round trip)
+    if ((++pops & 63) == 0 && *(volatile int32_t*)&a.flags[1] == 0) break;
     --sp;
     const int2 ent = stk[sp];
     __syncwarp();
