@@ -43,6 +43,9 @@ namespace egg {
 #ifndef EGG_UNROLL_G
 #define EGG_UNROLL_G 1
 #endif
+#ifndef EGG_PRED_ACC
+#define EGG_PRED_ACC 0
+#endif
 #ifndef EGG_UPD_MINB
 #define EGG_UPD_MINB 1
 #endif
@@ -301,6 +304,10 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
   bool act[kP];
 #pragma unroll
   for (int k = 0; k < kP; ++k) act[k] = (pm >> (k * 32 + lane)) & 1ull;
+  // points not active in this bucket get |q|^2 = 3e38: their distance is never within a limit
+  float ppa[kP];
+#pragma unroll
+  for (int k = 0; k < kP; ++k) ppa[k] = act[k] ? L.pp[k] : 3.0e38f;
   if constexpr (CNT) {
     wc.staged += cntc;
     wc.cls += (long long)cntc * popc64(pm);
@@ -335,14 +342,14 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
     bool any_pa = false, any_in = false;
 #pragma unroll
     for (int k = 0; k < kP; ++k) {
-      float a0 = L.pp[k] + cb[D], a1 = 0.f;
+      float a0 = ppa[k] + cb[D], a1 = 0.f;
 #pragma unroll
       for (int i = 0; i < D; i += 2) a0 = fmaf(L.q[k][i], cb[i], a0);
 #pragma unroll
       for (int i = 1; i < D; i += 2) a1 = fmaf(L.q[k][i], cb[i], a1);
       const float d2 = a0 + a1;
-      in[k] = act[k] && d2 <= cb[D + 1];
-      pa[k] = act[k] && !in[k] && d2 <= cb[D + 2];
+      in[k] = d2 <= cb[D + 1];
+      pa[k] = !in[k] && d2 <= cb[D + 2];
       any_pa |= pa[k];
       any_in |= in[k];
     }
@@ -399,6 +406,16 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
       }
 #pragma unroll
       for (int k = 0; k < kP; ++k) {
+#if EGG_PRED_ACC
+        if (in[k]) {  // predicated adds (no mask multiply)
+#pragma unroll
+          for (int i = 0; i < D; ++i) {
+            L.S[k][i] += sb[i];
+            L.C[k][i] += sb[D + i];
+          }
+          L.N[k] += cg;
+        }
+#else
         const float f = in[k] ? 1.f : 0.f;
 #pragma unroll
         for (int i = 0; i < D; ++i) {
@@ -406,6 +423,7 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
           L.C[k][i] = fmaf(f, sb[D + i], L.C[k][i]);
         }
         L.N[k] += in[k] ? cg : 0;
+#endif
       }
     }
   }
