@@ -290,8 +290,9 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
     const float emr = em * (1.f - 4.f * kU);
     const float ep = (a.e + rad) * (1.f + 4.f * kU);
     dst[D] = cc;
-    dst[D + 1] = em > 0.f ? emr * emr - gerr : -1.f;
-    dst[D + 2] = ep * ep + gerr;
+    // limits on |q|^2 - 2 q.c' (= d^2 - |c'|^2): |c'|^2 folded in, saving an add per point
+    dst[D + 1] = (em > 0.f ? emr * emr - gerr : -1.f) - cc;
+    dst[D + 2] = ep * ep + gerr - cc;
 #pragma unroll
     for (int i = 0; i < D; ++i) {
       dst[KA + i] = r[D + 3 + i];
@@ -342,7 +343,7 @@ __device__ __forceinline__ void stage_round(const UpdArgs<D>& a, Lane<D>& L, int
     bool any_pa = false, any_in = false;
 #pragma unroll
     for (int k = 0; k < kP; ++k) {
-      float a0 = ppa[k] + cb[D], a1 = 0.f;
+      float a0 = ppa[k], a1 = 0.f;
 #pragma unroll
       for (int i = 0; i < D; i += 2) a0 = fmaf(L.q[k][i], cb[i], a0);
 #pragma unroll
