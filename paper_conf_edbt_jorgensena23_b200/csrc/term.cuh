@@ -24,9 +24,10 @@ struct TermArgs {
   const uint32_t* __restrict__ g_hi;
   const int4* __restrict__ t_meta;
   const float* __restrict__ t_box;
+  const float* __restrict__ c_rec;  // unit centre + radius (cheap sphere pre-test)
   int64_t n, cap, lo, hi;
-  int32_t nc, stack_len;
-  float e2f, ed2f, rel;
+  int32_t nc, stack_len, bucket;
+  float e2f, ed2f, edf, rel;
   double e2d, ed2d;
   int32_t* flags;  // [1] second term AND, [3] error
 };
@@ -92,7 +93,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_second(const TermArgs<D> 
       pm = __ballot_sync(FULLMASK, act && mind <= lim_ed);
       if (pm == 0u) continue;
       const int4 meta = a.t_meta[ent.x];
-      if (meta.y - meta.x + 1 > kBucket) {
+      if (meta.y - meta.x + 1 > a.bucket) {
         if (sp + 2 > a.stack_len) {
           if (lane == 0) atomicExch(&a.flags[3], 1);
           break;
@@ -110,6 +111,17 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_second(const TermArgs<D> 
     }
     const bool pact = (pm >> lane) & 1u;
     for (int32_t c = first; c <= last; ++c) {
+      {  // sphere pre-test on the unit record: skip when |p - centre| - r > eps + delta
+        const float* __restrict__ rc = a.c_rec + (int64_t)c * CellRec<D>::kFloats;
+        float dc = 0.f;
+#pragma unroll
+        for (int i = 0; i < D; ++i) {
+          const float t = rc[i] - p[i];
+          dc = fmaf(t, t, dc);
+        }
+        const float reach = (a.edf + rc[D]) * (1.f + 4.f * kU);
+        if (!__any_sync(FULLMASK, pact && dc <= reach * reach * (1.f + a.rel))) continue;
+      }
       const int32_t gc = a.u2co ? a.u2co[c] : c;
       // prune the unit by its own MBR (no point of it within eps + delta)
       float umin = 0.f;
@@ -177,14 +189,18 @@ int run_second_term(Workspace& ws, int64_t lo, int64_t hi) {
   a.g_hi = ws.g_hi;
   a.t_meta = ws.t_meta;
   a.t_box = ws.t_box;
+  a.c_rec = ws.c_rec;
   a.n = ws.n;
   a.cap = ws.cap;
   a.lo = lo;
   a.hi = hi;
   a.nc = ws.n_cells;
   a.stack_len = ws.k.keybits + 4;
+  // as in the update: mostly-singleton units make subtree boxes useless for pruning
+  a.bucket = (int64_t)ws.n_cells * 2 > ws.n ? 256 : kBucket;
   a.e2f = ws.k.e2f;
   a.ed2f = ws.k.ed2f;
+  a.edf = ws.k.edf;
   a.rel = ws.k.rel;
   a.e2d = ws.k.e2;
   a.ed2d = ws.k.ed2;
