@@ -28,6 +28,8 @@
 // margin; point pairs inside the margin are re-decided in fp64 exactly as the
 // oracle's sum_i (q_i - p_i)^2 <= eps^2 (dimension order, no FMA).
 #pragma once
+#include <cstdlib>
+
 #include "common.cuh"
 
 namespace egg {
@@ -700,6 +702,8 @@ int run_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   // mostly-singleton cells (early iterations): subtree boxes rarely prune or cover, so
   // process bigger buckets; dense cells: descend further and let box tests prune / cover
   a.bucket = (int64_t)ws.n_cells * 2 > ws.n ? EGG_UPD_BUCKET_SPARSE : EGG_UPD_BUCKET_DENSE;
+  if (const char* e = getenv("EGGSYNC_BUCKET_SPARSE"); e && (int64_t)ws.n_cells * 2 > ws.n) a.bucket = atoi(e);
+  if (const char* e = getenv("EGGSYNC_BUCKET_DENSE"); e && (int64_t)ws.n_cells * 2 <= ws.n) a.bucket = atoi(e);
   a.e = ws.k.ef;
   a.e2f = ws.k.e2f;
   a.rel = ws.k.rel;
