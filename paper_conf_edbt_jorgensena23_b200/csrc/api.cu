@@ -124,6 +124,59 @@ static void cache_give(int device, char* p, size_t bytes, int32_t* hflags) {
   g_cache.push_back({device, p, bytes, hflags});
 }
 
+// grow-only range lists of the tensor-core update, cached per device like the arenas
+struct CachedRanges {
+  int device;
+  int2* p;
+  size_t cap;
+};
+static std::vector<CachedRanges> g_rcache;
+
+int tc_ranges_reserve(Workspace& ws, size_t need) {
+  if (ws.tc_rcap >= need) return EGGSYNC_OK;
+  {
+    std::lock_guard<std::mutex> lk(g_cache_mu);
+    for (size_t k = 0; k < g_rcache.size(); ++k) {
+      if (g_rcache[k].device == ws.cur_device && g_rcache[k].cap >= need) {
+        if (ws.tc_ranges) {
+          cudaStreamSynchronize(ws.stream);
+          cudaFree(ws.tc_ranges);
+        }
+        ws.tc_ranges = g_rcache[k].p;
+        ws.tc_rcap = g_rcache[k].cap;
+        g_rcache.erase(g_rcache.begin() + k);
+        return EGGSYNC_OK;
+      }
+    }
+  }
+  if (ws.tc_ranges) {
+    EGG_CUDA(cudaStreamSynchronize(ws.stream));
+    EGG_CUDA(cudaFree(ws.tc_ranges));
+    ws.tc_ranges = nullptr;
+    ws.tc_rcap = 0;
+  }
+  const size_t cap = need + need / 4 + 1024;
+  EGG_CUDA(cudaMalloc((void**)&ws.tc_ranges, cap * sizeof(int2)));
+  ws.tc_rcap = cap;
+  return EGGSYNC_OK;
+}
+
+static void tc_ranges_give(int device, int2* p, size_t cap) {
+  std::lock_guard<std::mutex> lk(g_cache_mu);
+  for (size_t k = 0; k < g_rcache.size(); ++k) {
+    if (g_rcache[k].device == device) {
+      if (g_rcache[k].cap >= cap) {
+        cudaFree(p);
+        return;
+      }
+      cudaFree(g_rcache[k].p);
+      g_rcache.erase(g_rcache.begin() + k);
+      break;
+    }
+  }
+  g_rcache.push_back({device, p, cap});
+}
+
 static void cache_clear() {
   std::lock_guard<std::mutex> lk(g_cache_mu);
   int prev = -1;
@@ -134,6 +187,11 @@ static void cache_clear() {
     cudaFreeHost(c.hflags);
   }
   g_cache.clear();
+  for (auto& c : g_rcache) {
+    cudaSetDevice(c.device);
+    cudaFree(c.p);
+  }
+  g_rcache.clear();
   if (prev >= 0) cudaSetDevice(prev);
 }
 
@@ -195,6 +253,11 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
       {(void**)&lab_final, sizeof(int32_t) * n},
       {(void**)&work, sizeof(unsigned long long) * 8},
       {(void**)&co_of, sizeof(int32_t) * n},
+      {(void**)&full_S, d <= 16 ? sizeof(double) * 2 * d * n : 0},
+      {(void**)&full_N, sizeof(int32_t) * n},
+      {(void**)&tc_nr, sizeof(int32_t) * (n / 128 + 2)},
+      {(void**)&tc_ne, sizeof(int32_t) * (n / 128 + 2)},
+      {(void**)&tc_roff, sizeof(int32_t) * (n / 128 + 2)},
       {(void**)&co_start, sizeof(int32_t) * (cap + 1)},
       {(void**)&co_cnt, sizeof(int32_t) * cap},
       {(void**)&co_lo, sizeof(uint32_t) * d * cap},
@@ -247,6 +310,9 @@ void Workspace::release() {
     if (stream) cudaStreamSynchronize(stream);  // no pending work may touch a cached arena
     cache_give(cur_device, arena, (size_t)bytes, h_flags);
   }
+  if (tc_ranges) tc_ranges_give(cur_device, tc_ranges, tc_rcap);
+  tc_ranges = nullptr;
+  tc_rcap = 0;
   arena = nullptr;
   h_flags = nullptr;
   if (own_stream && stream) cudaStreamDestroy(stream);
@@ -315,7 +381,7 @@ __global__ void k_unpack_owned(const float* __restrict__ g, int64_t n, int d, in
   if (pos < n) xs[(int64_t)i * n + pos] = g[t];
 }
 
-static int64_t owned_block_points(const Workspace& ws) { return 32 * (ws.d <= 12 ? 2 : 1); }  // = 32*ppl_for(d)
+static int64_t owned_block_points(const Workspace&) { return kOwnBlock; }
 static int64_t owned_count(const Workspace& ws, int32_t R) {
   const int64_t B = owned_block_points(ws);
   const int64_t nb = (ws.n + B - 1) / B;

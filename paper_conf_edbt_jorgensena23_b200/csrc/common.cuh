@@ -14,7 +14,8 @@ namespace egg {
 constexpr int kMaxD = EGGSYNC_MAX_D;
 constexpr int kMaxKeyWords = 8;  // Morton keys up to 512 bits (d * ceil(log2 w))
 constexpr int kWarpsPerCta = 4;  // update / second-term CTAs: 4 independent warps
-constexpr int kBucket = 32;      // subtree of <= kBucket cells is processed cell by cell
+constexpr int kBucket = 32;
+constexpr int kOwnBlock = 128;  // points per ownership block (multi-GPU interleave) = tensor-core tile      // subtree of <= kBucket cells is processed cell by cell
 constexpr uint32_t kLeafBit = 0x80000000u;
 constexpr float kU = 5.9604644775390625e-08f;  // 2^-24, fp32 unit roundoff
 
@@ -213,6 +214,16 @@ struct Workspace {
   bool count_work = false;
   int64_t launches = 0;  // kernel launches issued on this workspace (CUB internals counted by pass)
   int32_t own_stride = 1, own_offset = 0;  // block-interleaved ownership of the next update
+  // tensor-core update (update_tc.cuh): plan-pass outputs
+  double* full_S = nullptr;     // [2d][n] per-point sums of subtrees added whole (sorted order)
+  int32_t* full_N = nullptr;    // [n]
+  int32_t* tc_nr = nullptr;     // [tiles+1] ranges per point tile
+  int32_t* tc_ne = nullptr;     // [tiles+1] entries per point tile
+  int32_t* tc_roff = nullptr;   // [tiles+1] first range of each tile
+  int2* tc_ranges = nullptr;    // (first unit, count), grown on demand (process cache)
+  size_t tc_rcap = 0;
+  int tc_used = 0;              // 1 when the last update ran on the tensor cores
+  long long tc_pairs = 0;       // (point, entry) pairs classified by the last tensor-core update
 
   int alloc(int64_t n, int d, float eps, int device, cudaStream_t stream);
   void release();
@@ -227,6 +238,8 @@ int stage_second_term(Workspace& ws, int64_t lo, int64_t hi);
 int stage_labels(Workspace& ws, int32_t* labels_dev);  // labels of current cells, original order
 int stage_coords(Workspace& ws, int which, float* out_dev);  // row-major, original order
 int stage_scatter_i32(Workspace& ws, const int32_t* sorted_vals, int32_t* out_dev);
+
+int tc_ranges_reserve(Workspace& ws, size_t need);  // grow ws.tc_ranges to >= need entries
 
 // dispatch helpers (templated on D in update.cu / term.cu / grid.cu)
 int launch_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr_sorted);

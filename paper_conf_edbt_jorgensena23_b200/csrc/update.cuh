@@ -479,7 +479,10 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(cons
   double* mst = reinterpret_cast<double*>(wbase + W::off_mst());
   int4* stk = reinterpret_cast<int4*>(wbase + W::off_stk());
 
-  const int64_t base = a.lo + (((int64_t)blockIdx.x * kWarpsPerCta + wid) * a.stride + a.offset) * (32 * kP);
+  // ownership blocks of kOwnBlock points (b % stride == offset), each split into warp blocks
+  constexpr int kSub = kOwnBlock / (32 * kP);
+  const int64_t g = (int64_t)blockIdx.x * kWarpsPerCta + wid;
+  const int64_t base = a.lo + ((g / kSub) * a.stride + a.offset) * kOwnBlock + (g % kSub) * (32 * kP);
   Lane<D> L;
   unsigned long long amask = 0ull;
 #pragma unroll
@@ -677,7 +680,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(cons
 }
 
 template <int D>
-int run_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
+int run_update_simt(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   if (hi <= lo) return EGGSYNC_OK;
   UpdArgs<D> a;
   a.xs = ws.xs[ws.xcur];
@@ -719,11 +722,11 @@ int run_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   // block-interleaved ownership (multi-GPU load balance): blocks b with b % stride == offset
   a.stride = ws.own_stride;
   a.offset = ws.own_offset;
-  const int64_t B = 32 * PPL<D>::v;
-  const int64_t nblocks = (hi - lo + B - 1) / B;
+  const int64_t nblocks = (hi - lo + kOwnBlock - 1) / kOwnBlock;
   const int64_t owned = nblocks > a.offset ? (nblocks - a.offset + a.stride - 1) / a.stride : 0;
   if (owned == 0) return EGGSYNC_OK;
-  const unsigned grid = (unsigned)((owned + kWarpsPerCta - 1) / kWarpsPerCta);
+  const int64_t warps = owned * (kOwnBlock / (32 * PPL<D>::v));
+  const unsigned grid = (unsigned)((warps + kWarpsPerCta - 1) / kWarpsPerCta);
   kern<<<grid, kWarpsPerCta * 32, smem, ws.stream>>>(a);
   ws.launches += 1;
   EGG_CUDA(cudaGetLastError());

@@ -1,6 +1,7 @@
 // update_inst_3.cu -- explicit instantiations of the update and second-term kernels, D=25..32.
 // (split across files so the 32 dimension variants compile in parallel)
 #include "term.cuh"
+#include "update_tc.cuh"
 namespace egg {
 #if !defined(EGG_DEV_D) || EGG_DEV_D == 25
 template int run_update<25>(Workspace&, int64_t, int64_t, int32_t*);
