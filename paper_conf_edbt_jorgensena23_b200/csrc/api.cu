@@ -257,7 +257,8 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
       {(void**)&full_N, sizeof(int32_t) * n},
       {(void**)&tc_nr, sizeof(int32_t) * (n / 128 + 2)},
       {(void**)&tc_ne, sizeof(int32_t) * (n / 128 + 2)},
-      {(void**)&tc_roff, sizeof(int32_t) * (n / 128 + 2)},
+      {(void**)&tc_chunks, d <= 16 ? sizeof(int32_t) * (n / 128 + 2) * kChunkMax : 0},
+      {(void**)&tc_ctr, sizeof(int32_t) * 4},
       {(void**)&co_start, sizeof(int32_t) * (cap + 1)},
       {(void**)&co_cnt, sizeof(int32_t) * cap},
       {(void**)&co_lo, sizeof(uint32_t) * d * cap},

@@ -14,8 +14,10 @@ namespace egg {
 constexpr int kMaxD = EGGSYNC_MAX_D;
 constexpr int kMaxKeyWords = 8;  // Morton keys up to 512 bits (d * ceil(log2 w))
 constexpr int kWarpsPerCta = 4;  // update / second-term CTAs: 4 independent warps
-constexpr int kBucket = 32;
-constexpr int kOwnBlock = 128;  // points per ownership block (multi-GPU interleave) = tensor-core tile      // subtree of <= kBucket cells is processed cell by cell
+constexpr int kBucket = 32;      // subtree of <= kBucket cells is processed cell by cell
+constexpr int kOwnBlock = 128;  // points per ownership block (multi-GPU interleave) = tensor-core tile
+constexpr int kRangeChunk = 64;   // tensor-core plan: ranges are allocated in chunks of 64 ...
+constexpr int kChunkMax = 256;    // ... at most 256 chunks (16384 ranges) per point tile
 constexpr uint32_t kLeafBit = 0x80000000u;
 constexpr float kU = 5.9604644775390625e-08f;  // 2^-24, fp32 unit roundoff
 
@@ -219,7 +221,8 @@ struct Workspace {
   int32_t* full_N = nullptr;    // [n]
   int32_t* tc_nr = nullptr;     // [tiles+1] ranges per point tile
   int32_t* tc_ne = nullptr;     // [tiles+1] entries per point tile
-  int32_t* tc_roff = nullptr;   // [tiles+1] first range of each tile
+  int32_t* tc_chunks = nullptr; // [tiles][kChunkMax] first range of each chunk of a tile's range list
+  int32_t* tc_ctr = nullptr;    // [4] ranges allocated, chunk-table overflow
   int2* tc_ranges = nullptr;    // (first unit, count), grown on demand (process cache)
   size_t tc_rcap = 0;
   int tc_used = 0;              // 1 when the last update ran on the tensor cores

@@ -87,9 +87,12 @@ struct TcCfg {
 // Plan pass: one warp per 128-point tile (4 points per lane: row t = 32k + lane), warp-packet
 // traversal of the cell hierarchy with the per-point box tests of k_update.  A node that some
 // active point sees partially is descended (its full points stay active: they will classify
-// the cells exactly); a node nobody sees partially is added by its full points here; a subtree
-// of <= bucket cells that some point sees partially becomes a range of entries.
-// FILL=false counts ranges / entries per tile; FILL=true writes them and the full sums.
+// the cells exactly); a node nobody sees partially is added by its full points here (into
+// full_S / full_N, owned exclusively by the point's lane); a subtree of <= bucket cells that
+// some point sees partially becomes a range of entries.  One pass: a tile's ranges go into
+// chunks of kRangeChunk slots allocated from a global counter (chunk table per tile), so
+// no count pass / scan is needed.  Overflow of the range buffer or of the chunk table is
+// reported in ctr[0] / ctr[1] (the host grows the buffer and re-plans, or falls back).
 // ----------------------------------------------------------------------------------------
 template <int D>
 struct PlanArgs {
@@ -103,26 +106,22 @@ struct PlanArgs {
   float e;
   int32_t* t_nr;              // [ntiles] ranges per tile
   int32_t* t_ne;              // [ntiles] entries per tile
-  const int32_t* t_roff;      // [ntiles] first range of the tile (FILL)
-  int2* ranges;               // (first cell, count) (FILL)
-  double* full_S;             // [2D][n] (FILL)
-  int32_t* full_N;            // [n] (FILL)
+  int32_t* chunks;            // [ntiles][kChunkMax] first slot of each chunk
+  int32_t* ctr;               // [0] slots allocated, [1] chunk-table overflow
+  int64_t rcap;               // capacity of ranges
+  int2* ranges;               // (first cell, count)
+  double* full_S;             // [2D][n]
+  int32_t* full_N;            // [n]
   int32_t* flags;
 };
 
-constexpr int kPlanWarps = 2;
-
-template <int D>
-struct PlanSmem {
-  static constexpr int kMst = 4 * 2 * D * 32;  // doubles
-  __host__ __device__ static size_t bytes(int stack_len) { return (size_t)kMst * 8 + (size_t)stack_len * 32; }
-};
+constexpr int kPlanWarps = 4;
 
 __device__ __forceinline__ int64_t tc_tile_base(int64_t lo, int64_t tile, int32_t stride, int32_t offset) {
   return lo + (tile * stride + offset) * (int64_t)kTcTile;
 }
 
-template <int D, bool FILL>
+template <int D>
 __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a) {
   constexpr int kP = 4;
   constexpr int BS = ceil4(2 * D);
@@ -130,9 +129,7 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
   const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int64_t tile = (int64_t)blockIdx.x * kPlanWarps + wid;
   if (tile >= a.ntiles) return;
-  unsigned char* wb = psm + (size_t)wid * PlanSmem<D>::bytes(a.stack_len);
-  double* mst = reinterpret_cast<double*>(wb);  // [k][2D][32]
-  int* stk = reinterpret_cast<int*>(wb + PlanSmem<D>::kMst * 8);  // [stack_len][8]: node, m0..m3
+  int* stk = reinterpret_cast<int*>(psm) + (size_t)wid * a.stack_len * 8;  // [stack_len][8]: node, m0..m3
 
   const int64_t base = tc_tile_base(a.lo, tile, a.stride, a.offset);
   float q[kP][D];
@@ -179,11 +176,29 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
   const float nfu = fmaxf(a.e * (1.f - 4.f * kU) - slack, 0.f);
   const float lim_out = nlo * nlo * (1.f + (float)(2 * D + 8) * kU);
   const float lim_full = nfu * nfu * (1.f - (float)(2 * D + 8) * kU);
-  if constexpr (FILL)
-    for (int t = lane; t < PlanSmem<D>::kMst; t += 32) mst[t] = 0.0;
+  bool touched[kP] = {false, false, false, false};  // full_S of the point initialised
   int N[kP] = {0, 0, 0, 0};
   int32_t nr = 0, ne = 0;
-  int64_t rout = FILL ? a.t_roff[tile] : 0;
+  int32_t cbase = 0;  // first slot of the current chunk (warp-uniform)
+  int32_t* __restrict__ tch = a.chunks + tile * kChunkMax;
+  // append a range (warp-uniform call)
+  auto push = [&](int32_t first, int32_t cnt) {
+    const int32_t slot = nr % kRangeChunk;
+    if (slot == 0) {
+      int32_t b = 0;
+      if (lane == 0) {
+        b = atomicAdd(&a.ctr[0], kRangeChunk);
+        const int32_t ci = nr / kRangeChunk;
+        if (ci < kChunkMax) tch[ci] = b;
+        else atomicExch(&a.ctr[1], 1);
+      }
+      cbase = __shfl_sync(FULLMASK, b, 0);
+    }
+    if (lane == 0 && (int64_t)cbase + slot < a.rcap && nr < kChunkMax * kRangeChunk)
+      a.ranges[cbase + slot] = make_int2(first, cnt);
+    ++nr;
+    ne += cnt;
+  };
   __syncwarp();
   if (lane == 0) {
     stk[0] = a.nc > 1 ? 0 : (int)kLeafBit;
@@ -200,12 +215,7 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
     for (int k = 0; k < kP; ++k) m[k] = (uint32_t)stk[sp * 8 + 1 + k];
     __syncwarp();
     if (node & (int)kLeafBit) {  // a single cell: always an entry
-      if (lane == 0) {
-        if constexpr (FILL) a.ranges[rout] = make_int2(node & 0x7fffffff, 1);
-      }
-      ++rout;
-      ++nr;
-      ne += 1;
+      push(node & 0x7fffffff, 1);
       continue;
     }
     const float* __restrict__ bx = a.t_box + (int64_t)node * BS;
@@ -246,10 +256,12 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
         for (int k = 0; k < kP; ++k) {
           if (full[k]) {
             N[k] += cnt;
-            if constexpr (FILL) {
 #pragma unroll
-              for (int i = 0; i < 2 * D; ++i) mst[(k * 2 * D + i) * 32 + lane] += (double)sm[i];
+            for (int i = 0; i < 2 * D; ++i) {
+              double* dst = a.full_S + (int64_t)i * a.n + j[k];
+              *dst = (touched[k] ? *dst : 0.0) + (double)sm[i];
             }
+            touched[k] = true;
           }
         }
       }
@@ -258,12 +270,7 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
     const int4 meta = a.t_meta[node];
     const int ncell = meta.y - meta.x + 1;
     if (ncell <= a.bucket) {
-      if (lane == 0) {
-        if constexpr (FILL) a.ranges[rout] = make_int2(meta.x, ncell);
-      }
-      ++rout;
-      ++nr;
-      ne += ncell;
+      push(meta.x, ncell);
       continue;
     }
     if (sp + 2 > a.stack_len) {
@@ -282,19 +289,18 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
     sp += 2;
     __syncwarp();
   }
-  if constexpr (!FILL) {
-    if (lane == 0) {
-      a.t_nr[tile] = nr;
-      a.t_ne[tile] = ne;
-    }
-  } else {
+  if (lane == 0) {
+    a.t_nr[tile] = nr;
+    a.t_ne[tile] = ne;
+  }
 #pragma unroll
-    for (int k = 0; k < kP; ++k) {
-      if (valid[k]) {
+  for (int k = 0; k < kP; ++k) {
+    if (valid[k]) {
+      if (!touched[k]) {
 #pragma unroll
-        for (int i = 0; i < 2 * D; ++i) a.full_S[(int64_t)i * a.n + j[k]] = mst[(k * 2 * D + i) * 32 + lane];
-        a.full_N[j[k]] = N[k];
+        for (int i = 0; i < 2 * D; ++i) a.full_S[(int64_t)i * a.n + j[k]] = 0.0;
       }
+      a.full_N[j[k]] = N[k];
     }
   }
 }
@@ -314,7 +320,7 @@ struct TcArgs {
   const uint32_t* __restrict__ c_lo;
   const uint32_t* __restrict__ c_hi;
   const int2* __restrict__ ranges;
-  const int32_t* __restrict__ t_roff;
+  const int32_t* __restrict__ chunks;
   const int32_t* __restrict__ t_nr;
   const int32_t* __restrict__ t_ne;
   const double* __restrict__ full_S;
@@ -578,7 +584,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
       tc::bar_init(&ms->raw_full[b], 1);
     }
     tc::bar_fence_init();
-    ms->cursor_r = (int32_t)a.t_roff[tile];
+    ms->cursor_r = 0;
     ms->cursor_off = 0;
   }
   if (wid == 11) tc::tmem_alloc<512>(&ms->tbase);
@@ -681,10 +687,12 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
     const int pt = tid - 256;  // 0..kProd-1
     const int pw = wid - 8;
     constexpr int R = C::R;
-    const int32_t r_end = (int32_t)(a.t_roff[tile] + a.t_nr[tile]);
+    const int32_t r_end = a.t_nr[tile];
+    const int32_t* __restrict__ tch = a.chunks + tile * kChunkMax;
+    auto rget = [&](int32_t r) { return a.ranges[tch[r / kRangeChunk] + (r % kRangeChunk)]; };
     const float Rq = ms->Rq, Rqi = ms->Rqi;
     int2 gpre = make_int2(0, 0);  // this thread's range of the next expansion (prefetched)
-    if (ms->cursor_r + pt < r_end) gpre = a.ranges[ms->cursor_r + pt];
+    if (ms->cursor_r + pt < r_end) gpre = rget(ms->cursor_r + pt);
     auto expand = [&](int sb) {
       int filled = 0, nvalid = 0, round = 0;
       while (filled < kTcEnt) {
@@ -692,7 +700,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
         const int32_t rr = ms->cursor_r, off0 = ms->cursor_off;
         int32_t first = 0, cnt = 0;
         if (rr + pt < r_end) {
-          const int2 g = round == 0 ? gpre : a.ranges[rr + pt];
+          const int2 g = round == 0 ? gpre : rget(rr + pt);
           first = g.x;
           cnt = g.y;
           if (pt == 0) {
@@ -745,7 +753,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
       if (pt == 0) bar_expect_tx(&ms->raw_full[sb], (uint32_t)nvalid * R * 4);
       // prefetch the first range of the next expansion
       gpre = make_int2(0, 0);
-      if (ms->cursor_r + pt < r_end) gpre = a.ranges[ms->cursor_r + pt];
+      if (ms->cursor_r + pt < r_end) gpre = rget(ms->cursor_r + pt);
     };
     if (T > 0) expand(0);
     unsigned long long pc[4] = {0, 0, 0, 0};
@@ -993,33 +1001,35 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     p.e = ws.k.ef;
     p.t_nr = ws.tc_nr;
     p.t_ne = ws.tc_ne;
-    p.t_roff = ws.tc_roff;
-    p.ranges = nullptr;
+    p.chunks = ws.tc_chunks;
+    p.ctr = ws.tc_ctr;
     p.full_S = ws.full_S;
     p.full_N = ws.full_N;
     p.flags = ws.flags;
-    const size_t psmem = (size_t)kPlanWarps * PlanSmem<D>::bytes(p.stack_len);
+    const size_t psmem = (size_t)kPlanWarps * p.stack_len * 8 * sizeof(int);
     const unsigned pgrid = (unsigned)((owned + kPlanWarps - 1) / kPlanWarps);
-    EGG_CUDA(cudaFuncSetAttribute(k_tc_plan<D, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)psmem));
-    EGG_CUDA(cudaFuncSetAttribute(k_tc_plan<D, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)psmem));
-    EGG_CUDA(cudaMemsetAsync(ws.tc_nr + owned, 0, sizeof(int32_t), ws.stream));
-    k_tc_plan<D, false><<<pgrid, kPlanWarps * 32, psmem, ws.stream>>>(p);
-    EGG_CUDA(cudaGetLastError());
-    size_t tmp = 0;
-    EGG_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, ws.tc_nr, ws.tc_roff, (int)owned + 1, ws.stream));
-    if (tmp > ws.cub_bytes) {
-      set_error("cub scratch too small for the tensor-core plan scan");
-      return EGGSYNC_ECUDA;
+    EGG_CUDA(cudaFuncSetAttribute(k_tc_plan<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)psmem));
+    // the range buffer keeps its size across updates (process cache); a first guess of
+    // 16 chunks per tile, grown and re-planned when the plan reports more
+    EGG_TRY(tc_ranges_reserve(ws, (size_t)owned * 16 * kRangeChunk));
+    int32_t hc[2] = {0, 0};
+    for (int attempt = 0; attempt < 2; ++attempt) {
+      p.ranges = ws.tc_ranges;
+      p.rcap = (int64_t)ws.tc_rcap;
+      EGG_CUDA(cudaMemsetAsync(ws.tc_ctr, 0, 2 * sizeof(int32_t), ws.stream));
+      k_tc_plan<D><<<pgrid, kPlanWarps * 32, psmem, ws.stream>>>(p);
+      EGG_CUDA(cudaGetLastError());
+      EGG_CUDA(cudaMemcpyAsync(hc, ws.tc_ctr, 2 * sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
+      EGG_CUDA(cudaStreamSynchronize(ws.stream));
+      ws.launches += 1;
+      if (hc[1] || (size_t)(uint32_t)hc[0] <= ws.tc_rcap) break;
+      EGG_TRY(tc_ranges_reserve(ws, (size_t)(uint32_t)hc[0]));
     }
-    EGG_CUDA(cub::DeviceScan::ExclusiveSum(ws.cub_tmp, tmp, ws.tc_nr, ws.tc_roff, (int)owned + 1, ws.stream));
-    int32_t total = 0;
-    EGG_CUDA(cudaMemcpyAsync(&total, ws.tc_roff + owned, sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
-    EGG_CUDA(cudaStreamSynchronize(ws.stream));
-    ws.launches += 4;
-    EGG_TRY(tc_ranges_reserve(ws, (size_t)total + 1));
-    p.ranges = ws.tc_ranges;
-    k_tc_plan<D, true><<<pgrid, kPlanWarps * 32, psmem, ws.stream>>>(p);
-    EGG_CUDA(cudaGetLastError());
+    if (hc[1] || (size_t)(uint32_t)hc[0] > ws.tc_rcap) {  // a tile with > kChunkMax chunks: SIMT kernel
+      ws.tc_used = 0;
+      return run_update_simt<D>(ws, lo, hi, nbr);
+    }
+    const int32_t total = hc[0];
 
     TcArgs<D> a;
     a.xs = ws.xs[ws.xcur];
@@ -1032,7 +1042,7 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     a.c_lo = ws.c_lo;
     a.c_hi = ws.c_hi;
     a.ranges = ws.tc_ranges;
-    a.t_roff = ws.tc_roff;
+    a.chunks = ws.tc_chunks;
     a.t_nr = ws.tc_nr;
     a.t_ne = ws.tc_ne;
     a.full_S = ws.full_S;
