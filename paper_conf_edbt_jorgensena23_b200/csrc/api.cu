@@ -124,48 +124,51 @@ static void cache_give(int device, char* p, size_t bytes, int32_t* hflags) {
   g_cache.push_back({device, p, bytes, hflags});
 }
 
-// grow-only range lists of the tensor-core update, cached per device like the arenas
-struct CachedRanges {
+// grow-only buffers of the tensor-core update (range lists, entry lists), cached per
+// (device, tag) across calls like the arenas
+struct CachedBuf {
   int device;
-  int2* p;
-  size_t cap;
+  int tag;
+  void* p;
+  size_t bytes;
 };
-static std::vector<CachedRanges> g_rcache;
+static std::vector<CachedBuf> g_rcache;
 
-int tc_ranges_reserve(Workspace& ws, size_t need) {
-  if (ws.tc_rcap >= need) return EGGSYNC_OK;
+static int buf_reserve(Workspace& ws, int tag, void** p, size_t* cap_bytes, size_t need_bytes) {
+  if (*cap_bytes >= need_bytes) return EGGSYNC_OK;
   {
     std::lock_guard<std::mutex> lk(g_cache_mu);
     for (size_t k = 0; k < g_rcache.size(); ++k) {
-      if (g_rcache[k].device == ws.cur_device && g_rcache[k].cap >= need) {
-        if (ws.tc_ranges) {
+      if (g_rcache[k].device == ws.cur_device && g_rcache[k].tag == tag && g_rcache[k].bytes >= need_bytes) {
+        if (*p) {
           cudaStreamSynchronize(ws.stream);
-          cudaFree(ws.tc_ranges);
+          cudaFree(*p);
         }
-        ws.tc_ranges = g_rcache[k].p;
-        ws.tc_rcap = g_rcache[k].cap;
+        *p = g_rcache[k].p;
+        *cap_bytes = g_rcache[k].bytes;
         g_rcache.erase(g_rcache.begin() + k);
         return EGGSYNC_OK;
       }
     }
   }
-  if (ws.tc_ranges) {
+  if (*p) {
     EGG_CUDA(cudaStreamSynchronize(ws.stream));
-    EGG_CUDA(cudaFree(ws.tc_ranges));
-    ws.tc_ranges = nullptr;
-    ws.tc_rcap = 0;
+    EGG_CUDA(cudaFree(*p));
+    *p = nullptr;
+    *cap_bytes = 0;
   }
-  const size_t cap = need + need / 4 + 1024;
-  EGG_CUDA(cudaMalloc((void**)&ws.tc_ranges, cap * sizeof(int2)));
-  ws.tc_rcap = cap;
+  const size_t cap = need_bytes + need_bytes / 4 + 4096;
+  EGG_CUDA(cudaMalloc(p, cap));
+  *cap_bytes = cap;
   return EGGSYNC_OK;
 }
 
-static void tc_ranges_give(int device, int2* p, size_t cap) {
+static void buf_give(int device, int tag, void* p, size_t bytes) {
+  if (!p) return;
   std::lock_guard<std::mutex> lk(g_cache_mu);
   for (size_t k = 0; k < g_rcache.size(); ++k) {
-    if (g_rcache[k].device == device) {
-      if (g_rcache[k].cap >= cap) {
+    if (g_rcache[k].device == device && g_rcache[k].tag == tag) {
+      if (g_rcache[k].bytes >= bytes) {
         cudaFree(p);
         return;
       }
@@ -174,7 +177,21 @@ static void tc_ranges_give(int device, int2* p, size_t cap) {
       break;
     }
   }
-  g_rcache.push_back({device, p, cap});
+  g_rcache.push_back({device, tag, p, bytes});
+}
+
+int tc_ranges_reserve(Workspace& ws, size_t need) {
+  size_t cb = ws.tc_rcap * sizeof(int2);
+  const int rc = buf_reserve(ws, 0, (void**)&ws.tc_ranges, &cb, need * sizeof(int2));
+  ws.tc_rcap = cb / sizeof(int2);
+  return rc;
+}
+
+int tc_ent_reserve(Workspace& ws, size_t need) {
+  size_t cb = ws.tc_ecap * sizeof(int32_t);
+  const int rc = buf_reserve(ws, 1, (void**)&ws.tc_ent, &cb, need * sizeof(int32_t));
+  ws.tc_ecap = cb / sizeof(int32_t);
+  return rc;
 }
 
 static void cache_clear() {
@@ -259,6 +276,8 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
       {(void**)&tc_ne, sizeof(int32_t) * (n / 128 + 2)},
       {(void**)&tc_chunks, d <= 16 ? sizeof(int32_t) * (n / 128 + 2) * kChunkMax : 0},
       {(void**)&tc_ctr, sizeof(int32_t) * 4},
+      {(void**)&tc_epad, sizeof(int32_t) * (n / 128 + 2)},
+      {(void**)&tc_eoff, sizeof(int32_t) * (n / 128 + 2)},
       {(void**)&co_start, sizeof(int32_t) * (cap + 1)},
       {(void**)&co_cnt, sizeof(int32_t) * cap},
       {(void**)&co_lo, sizeof(uint32_t) * d * cap},
@@ -311,9 +330,12 @@ void Workspace::release() {
     if (stream) cudaStreamSynchronize(stream);  // no pending work may touch a cached arena
     cache_give(cur_device, arena, (size_t)bytes, h_flags);
   }
-  if (tc_ranges) tc_ranges_give(cur_device, tc_ranges, tc_rcap);
+  buf_give(cur_device, 0, tc_ranges, tc_rcap * sizeof(int2));
+  buf_give(cur_device, 1, tc_ent, tc_ecap * sizeof(int32_t));
   tc_ranges = nullptr;
   tc_rcap = 0;
+  tc_ent = nullptr;
+  tc_ecap = 0;
   arena = nullptr;
   h_flags = nullptr;
   if (own_stream && stream) cudaStreamDestroy(stream);

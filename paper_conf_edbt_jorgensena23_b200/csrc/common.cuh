@@ -223,6 +223,10 @@ struct Workspace {
   int32_t* tc_ne = nullptr;     // [tiles+1] entries per point tile
   int32_t* tc_chunks = nullptr; // [tiles][kChunkMax] first range of each chunk of a tile's range list
   int32_t* tc_ctr = nullptr;    // [4] ranges allocated, chunk-table overflow
+  int32_t* tc_epad = nullptr;   // [tiles+1] entries per tile padded to whole entry tiles
+  int32_t* tc_eoff = nullptr;   // [tiles+1] first entry of each tile in tc_ent (exclusive scan)
+  int32_t* tc_ent = nullptr;    // unit (cell) of every entry slot, -1 = padding (grown on demand)
+  size_t tc_ecap = 0;
   int2* tc_ranges = nullptr;    // (first unit, count), grown on demand (process cache)
   size_t tc_rcap = 0;
   int tc_used = 0;              // 1 when the last update ran on the tensor cores
@@ -243,6 +247,7 @@ int stage_coords(Workspace& ws, int which, float* out_dev);  // row-major, origi
 int stage_scatter_i32(Workspace& ws, const int32_t* sorted_vals, int32_t* out_dev);
 
 int tc_ranges_reserve(Workspace& ws, size_t need);  // grow ws.tc_ranges to >= need entries
+int tc_ent_reserve(Workspace& ws, size_t need);     // grow ws.tc_ent to >= need entries
 
 // dispatch helpers (templated on D in update.cu / term.cu / grid.cu)
 int launch_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr_sorted);

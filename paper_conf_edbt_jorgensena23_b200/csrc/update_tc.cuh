@@ -41,8 +41,9 @@ namespace egg {
 
 constexpr int kTcTile = 128;  // points per tile (TMEM lanes, GEMM M)
 constexpr int kTcEnt = 128;   // entries per entry tile (GEMM1 N, GEMM2 K)
-constexpr int kTcThreads = 12 * 32;  // 3 warps per SM sub-partition: <= 168 registers
-constexpr int kProd = 96;  // producer threads (warps 8-10)
+constexpr int kTcThreads = 13 * 32;  // 8 classifier + 4 producer warps + 1 MMA warp (<= 128 registers)
+constexpr int kProd = 128;  // producer threads (warps 8-11): one entry slot each
+constexpr int kMmaWarp = 12;  // TMEM owner; its lane 0 issues the MMAs
 constexpr int kTcMaxD = 12;
 #ifndef EGG_TC_DRAIN
 #define EGG_TC_DRAIN 2
@@ -54,31 +55,36 @@ struct TcCfg {
   static constexpr int K1 = ((3 * D + 2) + 7) / 8 * 8;  // GEMM1 K: q_hi, q_lo, q_hi, 1, 1
   static constexpr int NV = 2 * D + 1;                  // sin, cos, count
   static constexpr int N2 = (2 * NV + 15) / 16 * 16;     // GEMM2 N: hi | lo
-  // TMEM columns
+  // TMEM columns: Q, NS S/P buffers (3 when they fit: GEMM1 runs ahead of both
+  // classifier groups), one O accumulator per classifier group
   static constexpr int kColQ = 0;
   static constexpr int kColS = K1;                  // S/P buffers: kColS + 128*b
-  static constexpr int kColO = K1 + 2 * kTcEnt;     // O buffers: kColO + N2*b
-  static_assert(kColO + 2 * N2 <= 512, "TMEM budget");
-  static constexpr int kLdO = (N2 + 31) / 32;       // 32-column loads per drain
-  static_assert(kColO + N2 + 32 * kLdO <= 512, "drain loads stay inside the allocation");
+#ifndef EGG_TC_NS
+#define EGG_TC_NS 3
+#endif
+  static constexpr int kNS0 = (EGG_TC_NS >= 3 && K1 + 3 * kTcEnt + 2 * N2 <= 512) ? 3 : 2;
+  static constexpr int kColO0 = K1 + kNS0 * kTcEnt;
+  static_assert(K1 + 2 * kTcEnt + 2 * N2 <= 512, "TMEM budget");
+  static_assert(N2 % 16 == 0, "drain loads of 16 columns");
   // shared-memory stage: B1 (K-major: entry rows), B2 (K-major: value rows), meta
   static constexpr int SBO1 = (K1 / 4) * 128;
   static constexpr int kB1Bytes = kTcEnt * K1 * 4;
   static constexpr int LBO2 = 144;  // 16-byte gap per 4-entry chunk: conflict-free producer stores
   static constexpr int SBO2 = (kTcEnt / 4) * LBO2;
   static constexpr int kB2Bytes = (N2 / 8) * SBO2;
-  static constexpr int kMetaBytes = kTcEnt * 16 + 16 + D * kTcEnt * 4;  // W, cnt, start, cell; Wmax[4]; xc[D][128]
+  static constexpr int kMetaBytes = kTcEnt * 16 + 16;  // W, cnt, start, cell; Wmax[4]
   static constexpr int kStageBytes = kB1Bytes + kB2Bytes + kMetaBytes;
   static constexpr int R = CellRec<D>::kFloats;
   static constexpr int kRawBytes = 2 * kTcEnt * R * 4;      // cell records staged by bulk copies [2][128][R]
-  static constexpr int kRareBytes = NV * kTcTile * 8;      // exact-path sums, fixed point [NV][row] (i64)
+  // per classifier group: exact fixed-point sums [NV][row] (rare-path count at 2D) + tensor-core count [row]
+  static constexpr int kRareBytes = 2 * (NV + 1) * kTcTile * 8;
   static constexpr int kMiscBytes = 3072;
   static constexpr int kBudget = 227 * 1024 - 1024;
   static constexpr int kStages =
       (kBudget - kRawBytes - kRareBytes - kMiscBytes) / kStageBytes >= 3 ? 3 : 2;
   static constexpr int kRingBytes = kStages * kStageBytes;
-  static constexpr int kXchBytes = NV * kTcTile * 8;  // epilogue exchange (reuses the ring)
-  static_assert(kXchBytes <= kRingBytes, "exchange fits the ring");
+  static constexpr int kNS = kNS0 < kStages ? kNS0 : kStages;  // the MMA loop needs stages >= S buffers
+  static constexpr int kColO = K1 + kNS * kTcEnt;   // O buffers: kColO + N2*g
   static constexpr size_t kSmem = (size_t)kRingBytes + kRawBytes + kRareBytes + kMiscBytes + 1024;  // +1024 align
   static_assert(kSmem <= 227 * 1024, "shared-memory budget");
 };
@@ -106,6 +112,7 @@ struct PlanArgs {
   float e;
   int32_t* t_nr;              // [ntiles] ranges per tile
   int32_t* t_ne;              // [ntiles] entries per tile
+  int32_t* t_epad;            // [ntiles] entries padded to whole entry tiles
   int32_t* chunks;            // [ntiles][kChunkMax] first slot of each chunk
   int32_t* ctr;               // [0] slots allocated, [1] chunk-table overflow
   int64_t rcap;               // capacity of ranges
@@ -292,6 +299,7 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
   if (lane == 0) {
     a.t_nr[tile] = nr;
     a.t_ne[tile] = ne;
+    a.t_epad[tile] = (ne + kTcEnt - 1) / kTcEnt * kTcEnt;
   }
 #pragma unroll
   for (int k = 0; k < kP; ++k) {
@@ -303,6 +311,44 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
       a.full_N[j[k]] = N[k];
     }
   }
+}
+
+// Expansion of each tile's range list into its entry-slot list (one warp per tile): slot e of
+// the tile holds the unit (cell) of entry e; the list is padded with -1 to whole entry tiles.
+template <int kUnused>
+__global__ void __launch_bounds__(128) k_tc_expand(const int2* __restrict__ ranges, const int32_t* __restrict__ chunks,
+                                                   const int32_t* __restrict__ t_nr, const int32_t* __restrict__ t_ne,
+                                                   const int32_t* __restrict__ eoff, int32_t* __restrict__ ent,
+                                                   int32_t ntiles) {
+  const int lane = threadIdx.x & 31;
+  const int64_t tile = (int64_t)blockIdx.x * 4 + (threadIdx.x >> 5);
+  if (tile >= ntiles) return;
+  const int32_t nr = t_nr[tile];
+  const int32_t* __restrict__ tch = chunks + tile * kChunkMax;
+  int32_t* __restrict__ out = ent + eoff[tile];
+  int32_t off = 0;
+  for (int32_t r0 = 0; r0 < nr; r0 += 32) {
+    const int32_t r = r0 + lane;
+    const int2 g = r < nr ? ranges[tch[r / kRangeChunk] + (r % kRangeChunk)] : make_int2(0, 0);
+    int32_t incl = g.y;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const int32_t u = __shfl_up_sync(FULLMASK, incl, o);
+      if (lane >= o) incl += u;
+    }
+    const int32_t excl = incl - g.y;
+    const int32_t tot = __shfl_sync(FULLMASK, incl, 31);
+    const int kn = min(32, nr - r0);
+    for (int k = 0; k < kn; ++k) {
+      const int32_t first = __shfl_sync(FULLMASK, g.x, k), cnt = __shfl_sync(FULLMASK, g.y, k),
+                    ex = __shfl_sync(FULLMASK, excl, k);
+      for (int32_t t = lane; t < cnt; t += 32) out[off + ex + t] = first + t;
+    }
+    off += tot;
+  }
+  const int32_t ne = t_ne[tile];
+  const int32_t padded = (ne + kTcEnt - 1) / kTcEnt * kTcEnt;
+  for (int32_t t = ne + lane; t < padded; t += 32) out[t] = -1;
 }
 
 // ----------------------------------------------------------------------------------------
@@ -319,9 +365,8 @@ struct TcArgs {
   const float* __restrict__ c_rec;
   const uint32_t* __restrict__ c_lo;
   const uint32_t* __restrict__ c_hi;
-  const int2* __restrict__ ranges;
-  const int32_t* __restrict__ chunks;
-  const int32_t* __restrict__ t_nr;
+  const int32_t* __restrict__ ent;   // unit of every entry slot (-1 = padding)
+  const int32_t* __restrict__ eoff;  // [ntiles] first slot of each point tile
   const int32_t* __restrict__ t_ne;
   const double* __restrict__ full_S;
   const int32_t* __restrict__ full_N;
@@ -340,28 +385,22 @@ __device__ __forceinline__ void named_bar(int id, int cnt) {
 
 // shared-memory header of the TC kernel
 struct TcMisc {
-  uint64_t stage_full[3], stage_empty[3], s_full[2], p_full[2], o_full[2], raw_full[2];
+  uint64_t stage_full[3], stage_empty[3], s_full[3], p_full[3], o_full[2];  // s_full / p_full: per S buffer
   uint32_t tbase;
-  int32_t cursor_r, cursor_off;
-  int32_t scan_w[4];  // producer warp totals
   float o[kTcMaxD], s0[kTcMaxD], c0[kTcMaxD];
   float lo[4][kTcMaxD], hi[4][kTcMaxD];
   float Rq, Rqi;
-  int32_t slot[2][kTcEnt];  // unit of each entry slot (-1: padding), double-buffered
 };
 static_assert(sizeof(TcMisc) <= 3072, "misc header");
 
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-          tc::smem_addr(dst)),
-      "l"(src), "r"(bytes), "r"(tc::smem_addr(bar))
-      : "memory");
+// per-thread asynchronous 16-byte global -> shared copies (L2 only), waited per thread
+__device__ __forceinline__ void cp_async16(void* dst, const void* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(tc::smem_addr(dst)), "l"(src) : "memory");
 }
-__device__ __forceinline__ void bar_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(tc::smem_addr(bar)), "r"(bytes)
-               : "memory");
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
 }
 
 template <int D>
@@ -373,7 +412,6 @@ struct TcStage {
   int32_t* start;
   int32_t* cell;
   float* wmax;
-  float* xc;  // [D][kTcEnt] unit centres (a single point's exact coordinates)
   __device__ TcStage(unsigned char* ring, int s) {
     using C = TcCfg<D>;
     unsigned char* p = ring + (size_t)s * C::kStageBytes;
@@ -385,16 +423,15 @@ struct TcStage {
     start = reinterpret_cast<int32_t*>(m + 8 * kTcEnt);
     cell = reinterpret_cast<int32_t*>(m + 12 * kTcEnt);
     wmax = reinterpret_cast<float*>(m + 16 * kTcEnt);
-    xc = reinterpret_cast<float*>(m + 16 * kTcEnt + 16);
   }
 };
 
 // Exact path for a multi-point unit e inside the band of point pe (P stays 0 for the pair):
 // refine with the unit's exact MBR, then its points one by one (fp32 + fp64 re-decision as
-// in k_update).  Sums go into the tile's fixed-point (2^-32) rare sums [NV][row] with
-// integer atomics: exact and independent of the order of the two classifier groups.
+// in k_update).  Sums go into the classifier group's own fixed-point (2^-32) sums [NV][row]:
+// exact, and the two groups' arrays are added in the epilogue (order-independent).
 __device__ __forceinline__ void rare_add(unsigned long long* rare, int i, int row, double v) {
-  atomicAdd(&rare[i * kTcTile + row], (unsigned long long)(long long)llrint(v * kFix));
+  rare[i * kTcTile + row] += (unsigned long long)llrint(v * kFix);  // the group's own row: no atomics
 }
 template <int D>
 __device__ __noinline__ void tc_rare(const TcArgs<D>& a, const float* __restrict__ pe, int e,
@@ -418,7 +455,7 @@ __device__ __noinline__ void tc_rare(const TcArgs<D>& a, const float* __restrict
     const float* __restrict__ r = a.c_rec + (int64_t)c * R;
 #pragma unroll
     for (int i = 0; i < 2 * D; ++i) rare_add(rare, i, row, (double)r[D + 3 + i]);
-    atomicAdd(&rare[2 * D * kTcTile + row], (unsigned long long)cnt);
+    rare[2 * D * kTcTile + row] += (unsigned long long)cnt;
     return;
   }
   unsigned long long nin = 0;
@@ -443,7 +480,7 @@ __device__ __noinline__ void tc_rare(const TcArgs<D>& a, const float* __restrict
       ++nin;
     }
   }
-  if (nin) atomicAdd(&rare[2 * D * kTcTile + row], nin);
+  rare[2 * D * kTcTile + row] += nin;
 }
 
 // Build entry slot `pt` (unit c, or padding when c < 0) of a stage: B1 row, B2 column, meta.
@@ -457,7 +494,6 @@ __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const TcMisc
   float b[K1];
   float vh[NV], vl[NV];
   float W = 0.f;
-  float xcv[D];
   int32_t ccnt = 0, cstart = 0;
   if (c >= 0) {
     float r[R];
@@ -473,7 +509,6 @@ __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const TcMisc
     float cc = 0.f, cinf = 0.f;
 #pragma unroll
     for (int i = 0; i < D; ++i) {
-      xcv[i] = r[i];
       const float cp = r[i] - ms->o[i];
       const float h = tc::tf32_hi(cp);
       b[i] = -2.f * h;
@@ -517,7 +552,6 @@ __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const TcMisc
     for (int k = 0; k < 3 * D + 2; ++k) b[k] = 0.f;
     b[3 * D] = 1073741824.f;  // v = 2^30: outside, never ambiguous
 #pragma unroll
-    for (int i = 0; i < D; ++i) xcv[i] = 0.f;
 #pragma unroll
     for (int k = 0; k < NV; ++k) vh[k] = vl[k] = 0.f;
     ccnt = 0;
@@ -544,9 +578,7 @@ __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const TcMisc
 #pragma unroll
     for (int n = 2 * NV; n < N2; ++n) *reinterpret_cast<float*>(b2 + (n >> 3) * C::SBO2 + (n & 7) * 16) = 0.f;
   }
-  st.W[pt] = W;
 #pragma unroll
-  for (int i = 0; i < D; ++i) st.xc[i * kTcEnt + pt] = xcv[i];
   st.cnt[pt] = ccnt;
   st.start[pt] = cstart;
   st.cell[pt] = c;
@@ -558,8 +590,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
   using C = TcCfg<D>;
   constexpr int K1 = C::K1, NV = C::NV, N2 = C::N2, NST = C::kStages;
   extern __shared__ __align__(16) unsigned char tsm_raw[];
-  unsigned char* tsm =
-      reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(tsm_raw) + 1023) & ~(uintptr_t)1023);
+  unsigned char* tsm = tsm_raw + ((1024u - (tc::smem_addr(tsm_raw) & 1023u)) & 1023u);
   unsigned char* ring = tsm;
   float* raw = reinterpret_cast<float*>(tsm + C::kRingBytes);  // [2][kTcEnt][R] staged cell records
   unsigned long long* rare = reinterpret_cast<unsigned long long*>(tsm + C::kRingBytes + C::kRawBytes);
@@ -569,7 +600,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
   const int64_t tile = blockIdx.x;
   const int64_t base = tc_tile_base(a.lo, tile, a.stride, a.offset);
   const int32_t ne = a.t_ne[tile];
-  const int T = (ne + kTcEnt - 1) / kTcEnt;
+  const int T = (ne + kTcEnt - 1) / kTcEnt;  // entry tiles (the slot list is padded to T * kTcEnt)
 
   // ---- setup -------------------------------------------------------------------------
   if (tid == 0) {
@@ -577,18 +608,15 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
       tc::bar_init(&ms->stage_full[s], kProd);
       tc::bar_init(&ms->stage_empty[s], 1);
     }
-    for (int b = 0; b < 2; ++b) {
+    for (int b = 0; b < C::kNS; ++b) {
       tc::bar_init(&ms->s_full[b], 1);
       tc::bar_init(&ms->p_full[b], kTcTile);
-      tc::bar_init(&ms->o_full[b], 1);
-      tc::bar_init(&ms->raw_full[b], 1);
     }
+    for (int b = 0; b < 2; ++b) tc::bar_init(&ms->o_full[b], 1);
     tc::bar_fence_init();
-    ms->cursor_r = 0;
-    ms->cursor_off = 0;
   }
-  if (wid == 11) tc::tmem_alloc<512>(&ms->tbase);
-  for (int t = tid; t < NV * kTcTile; t += kTcThreads) rare[t] = 0ull;
+  if (wid == kMmaWarp) tc::tmem_alloc<512>(&ms->tbase);
+  for (int t = tid; t < 2 * (NV + 1) * kTcTile; t += kTcThreads) rare[t] = 0ull;
 
   // classifier rows: every classifier thread holds its point
   const bool is_cls = wid < 8;
@@ -679,91 +707,45 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
   tc::fence_after();
   const uint32_t tb = ms->tbase;
 
-  if (wid >= 8 && wid < 11) {
+  if (wid >= 8 && wid < kMmaWarp) {
     // ================================ producers ================================
-    // Software pipeline: while entry tile jt is built from records already staged in
-    // raw[jt&1], the ranges of tile jt+1 are expanded into slots and their records are
-    // fetched by bulk copies (cp.async.bulk, mbarrier raw_full) into raw[(jt+1)&1].
+    // Thread pt owns entry slot pt of every entry tile.  While entry tile jt is built from
+    // the record staged in raw[jt&1][pt], the record of slot pt of tile jt+1 is fetched by
+    // asynchronous copies (cp.async, waited by the same thread: no cross-thread hand-off).
     const int pt = tid - 256;  // 0..kProd-1
     const int pw = wid - 8;
     constexpr int R = C::R;
-    const int32_t r_end = a.t_nr[tile];
-    const int32_t* __restrict__ tch = a.chunks + tile * kChunkMax;
-    auto rget = [&](int32_t r) { return a.ranges[tch[r / kRangeChunk] + (r % kRangeChunk)]; };
+    const int32_t* __restrict__ ent = a.ent + a.eoff[tile];
     const float Rq = ms->Rq, Rqi = ms->Rqi;
-    int2 gpre = make_int2(0, 0);  // this thread's range of the next expansion (prefetched)
-    if (ms->cursor_r + pt < r_end) gpre = rget(ms->cursor_r + pt);
-    auto expand = [&](int sb) {
-      int filled = 0, nvalid = 0, round = 0;
-      while (filled < kTcEnt) {
-        const int need = kTcEnt - filled;
-        const int32_t rr = ms->cursor_r, off0 = ms->cursor_off;
-        int32_t first = 0, cnt = 0;
-        if (rr + pt < r_end) {
-          const int2 g = round == 0 ? gpre : rget(rr + pt);
-          first = g.x;
-          cnt = g.y;
-          if (pt == 0) {
-            first += off0;
-            cnt -= off0;
-          }
-        }
-        int32_t incl = cnt;
+    // records of slot pt of the next entry tile are copied while this one is built; the
+    // slot's unit index is loaded one more tile ahead so its latency is hidden as well
+    auto fetch = [&](int32_t c, int sb) {
+      if (c >= 0) {
+        float* dst = raw + ((size_t)sb * kTcEnt + pt) * R;
+        const float* src = a.c_rec + (int64_t)c * R;
 #pragma unroll
-        for (int off = 1; off < 32; off <<= 1) {
-          const int32_t u = __shfl_up_sync(FULLMASK, incl, off);
-          if (lane >= off) incl += u;
-        }
-        if (lane == 31) ms->scan_w[pw] = incl;
-        named_bar(1, kProd);
-        int32_t wpre = 0, total = 0;
-#pragma unroll
-        for (int w = 0; w < kProd / 32; ++w) {
-          const int32_t x = ms->scan_w[w];
-          wpre += w < pw ? x : 0;
-          total += x;
-        }
-        incl += wpre;
-        const int32_t excl = incl - cnt;
-        const int32_t hi_ = min(incl, need);
-        if (excl < hi_) {  // slots [filled+excl, filled+hi_) <- units first.., one bulk copy
-          for (int32_t sl = excl; sl < hi_; ++sl) ms->slot[sb][filled + sl] = first + (sl - excl);
-          bulk_g2s(raw + ((size_t)sb * kTcEnt + filled + excl) * R, a.c_rec + (int64_t)first * R,
-                   (uint32_t)(hi_ - excl) * R * 4, &ms->raw_full[sb]);
-        }
-        // cursor of the next round / entry tile (every thread read the old one above)
-        if (excl < need && incl > need) {
-          ms->cursor_r = rr + pt;
-          ms->cursor_off = (pt == 0 ? off0 : 0) + (need - excl);
-        } else if (incl == need && cnt > 0) {
-          ms->cursor_r = rr + pt + 1;
-          ms->cursor_off = 0;
-        } else if (pt == 0 && total < need) {
-          ms->cursor_r = min(rr + kProd, r_end);
-          ms->cursor_off = 0;
-        }
-        const bool exhausted = total < need && rr + kProd >= r_end;
-        if (exhausted)
-          for (int sl = filled + total + pt; sl < kTcEnt; sl += kProd) ms->slot[sb][sl] = -1;
-        named_bar(1, kProd);
-        nvalid += min(total, need);
-        filled += exhausted ? need : min(total, need);
-        ++round;
+        for (int k = 0; k < R / 4; ++k) cp_async16(dst + 4 * k, src + 4 * k);
       }
-      if (pt == 0) bar_expect_tx(&ms->raw_full[sb], (uint32_t)nvalid * R * 4);
-      // prefetch the first range of the next expansion
-      gpre = make_int2(0, 0);
-      if (ms->cursor_r + pt < r_end) gpre = rget(ms->cursor_r + pt);
+      cp_async_commit();
     };
-    if (T > 0) expand(0);
+    auto unit_of = [&](int jt) -> int32_t { return jt < T ? ent[(int64_t)jt * kTcEnt + pt] : -1; };
+    int32_t c_cur = unit_of(0), c_nxt = unit_of(1);
+    if (T > 0) fetch(c_cur, 0);
     unsigned long long pc[4] = {0, 0, 0, 0};
     for (int jt = 0; jt < T; ++jt) {
       const int s = jt % NST, sb = jt & 1;
+      const int32_t c = c_cur;
       long long t0 = clock64();
-      if (jt + 1 < T) expand(sb ^ 1);
+      if (jt + 1 < T) {
+        fetch(c_nxt, sb ^ 1);
+        c_cur = c_nxt;
+        c_nxt = unit_of(jt + 2);
+        cp_async_wait<1>();
+      } else {
+        cp_async_wait<0>();
+      }
       long long t1 = clock64();
-      tc::bar_wait(&ms->raw_full[sb], (jt >> 1) & 1);
-      long long t2 = clock64();
+      long long t2 = t1;
       if (jt >= NST) tc::bar_wait(&ms->stage_empty[s], ((jt / NST) - 1) & 1);
       long long t3 = clock64();
       pc[0] += t1 - t0;
@@ -772,21 +754,11 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
       pc[3] -= t3;
       TcStage<D> st(ring, s);
       const float* rb = raw + (size_t)sb * kTcEnt * R;
-      {  // entries 0..95: warp pw builds chunk pw
-        const float W = tc_build_entry<D>(a, ms, st, pt, ms->slot[sb][pt], rb + pt * R, Rq, Rqi);
-        float wm = W;
+      const float W = tc_build_entry<D>(a, ms, st, pt, c, rb + pt * R, Rq, Rqi);
+      float wm = W;
 #pragma unroll
-        for (int off = 16; off > 0; off >>= 1) wm = fmaxf(wm, __shfl_xor_sync(FULLMASK, wm, off));
-        if (lane == 0) st.wmax[pw] = wm;
-      }
-      if (pw == 0) {  // entries 96..127: chunk 3
-        const int e = kProd + pt;
-        const float W = tc_build_entry<D>(a, ms, st, e, ms->slot[sb][e], rb + e * R, Rq, Rqi);
-        float wm = W;
-#pragma unroll
-        for (int off = 16; off > 0; off >>= 1) wm = fmaxf(wm, __shfl_xor_sync(FULLMASK, wm, off));
-        if (lane == 0) st.wmax[3] = wm;
-      }
+      for (int off = 16; off > 0; off >>= 1) wm = fmaxf(wm, __shfl_xor_sync(FULLMASK, wm, off));
+      if (lane == 0) st.wmax[pw] = wm;
       tc::fence_proxy_async();
       tc::bar_arrive(&ms->stage_full[s]);
       pc[3] += clock64();
@@ -795,82 +767,107 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
       for (int k = 0; k < 4; ++k) atomicAdd(&a.prof[k], pc[k]);
       atomicAdd(&a.prof[4], (unsigned long long)T);
     }
-  } else if (wid == 11) {
+  }
+
+  if (wid == kMmaWarp) {
     // ================================ MMA issue ================================
+    // One thread issues, in order (the tensor pipe executes them in order):
+    //   GEMM1(j1)  S[j1 % NS] = Q . B1(j1)^T      once stage j1 is built, and only after
+    //              GEMM2(j1 - NS) (the last reader of that S buffer) was issued
+    //   GEMM2(j2)  O[g] (+)= P . B2(j2)^T         once its classifier group wrote P
+    // polling both conditions, so neither kind waits behind the other.
     if (lane == 0) {
       constexpr uint32_t id1 = tc::idesc_tf32(128, kTcEnt, false);
       constexpr uint32_t id2 = tc::idesc_tf32(128, N2, false);
+      constexpr int NS = C::kNS;
       const uint32_t ring_s = tc::smem_addr(ring);
       const int T0 = (T + 1) / 2, T1 = T / 2;  // entry tiles of group 0 / 1
-      for (int jt = 0; jt <= T; ++jt) {
-        if (jt < T) {
-          const int s = jt % NST, bb = jt & 1;
-          tc::bar_wait(&ms->stage_full[s], (jt / NST) & 1);
+      int j1 = 0, j2 = 0;
+      while (j2 < T) {
+        bool did = false;
+        if (j1 < T && j1 - j2 < NS && tc::bar_test(&ms->stage_full[j1 % NST], (j1 / NST) & 1)) {
+          const int s = j1 % NST, sb = j1 % NS;
           tc::fence_after();
           const uint32_t b1 = ring_s + s * C::kStageBytes;
 #pragma unroll
           for (int k = 0; k < K1 / 8; ++k)
-            tc::mma_ts(tb + C::kColS + kTcEnt * bb, tb + C::kColQ + 8 * k, tc::sdesc(b1 + k * 256, 128, C::SBO1), id1,
+            tc::mma_ts(tb + C::kColS + kTcEnt * sb, tb + C::kColQ + 8 * k, tc::sdesc(b1 + k * 256, 128, C::SBO1), id1,
                        k > 0);
-          tc::mma_commit(&ms->s_full[bb]);
+          tc::mma_commit(&ms->s_full[sb]);
+          ++j1;
+          did = true;
         }
-        if (jt >= 1) {
-          const int jj = jt - 1, s = jj % NST, bb = jj & 1, kk = jj >> 1;
-          tc::bar_wait(&ms->p_full[bb], kk & 1);
+        if (j2 < j1 && tc::bar_test(&ms->p_full[j2 % NS], (j2 / NS) & 1)) {  // per S buffer: never two phases ahead
+          const int jj = j2, s = jj % NST, sb = jj % NS, g = jj & 1, kk = jj >> 1;
           tc::fence_after();
           const uint32_t b2 = ring_s + s * C::kStageBytes + C::kB1Bytes;
           const uint32_t acc0 = (kk % kDrain) != 0;
 #pragma unroll
           for (int k = 0; k < kTcEnt / 8; ++k)
-            tc::mma_ts(tb + C::kColO + N2 * bb, tb + C::kColS + kTcEnt * bb + 8 * k,
+            tc::mma_ts(tb + C::kColO + N2 * g, tb + C::kColS + kTcEnt * sb + 8 * k,
                        tc::sdesc(b2 + k * 2 * C::LBO2, C::LBO2, C::SBO2), id2, (k > 0) || acc0);
           tc::mma_commit(&ms->stage_empty[s]);
-          const int Tg = bb ? T1 : T0;
-          if ((kk % kDrain) == kDrain - 1 || kk == Tg - 1) tc::mma_commit(&ms->o_full[bb]);
+          const int Tg = g ? T1 : T0;
+          if ((kk % kDrain) == kDrain - 1 || kk == Tg - 1) tc::mma_commit(&ms->o_full[g]);
+          ++j2;
+          did = true;
         }
+        if (!did) __nanosleep(20);
       }
     }
     __syncwarp();
   }
 
-  double acc[NV];
-#pragma unroll
-  for (int i = 0; i < NV; ++i) acc[i] = 0.0;
   if (is_cls) {
     // ================================ classifiers ================================
     const uint32_t lane_off = (uint32_t)(32 * (wid & 3)) << 16;
     const int Tg = grp ? T / 2 : (T + 1) / 2;
+    unsigned long long* racc = rare + grp * (NV + 1) * kTcTile;  // this group's sums (rows are exclusive)
     int dc = 0;  // drains done
     unsigned long long cw[3] = {0, 0, 0};
+    // O (fp32, <= kDrain entry tiles) -> the row's exact fixed-point sums in shared memory
+    // (integer atomics: both groups add to the same rows, order-independent)
     auto drain = [&]() {
       tc::bar_wait(&ms->o_full[grp], dc & 1);
       ++dc;
       tc::fence_after();
+      double hi[NV];
 #pragma unroll
-      for (int c = 0; c < C::kLdO; ++c) {
-        uint32_t v[32];
-        tc::ld32(tb + lane_off + C::kColO + N2 * grp + 32 * c, v);
+      for (int c = 0; c < N2 / 16; ++c) {
+        uint32_t v[16];
+        tc::ld16(tb + lane_off + C::kColO + N2 * grp + 16 * c, v);
         tc::wait_ld();
 #pragma unroll
-        for (int jx = 0; jx < 32; ++jx) {
-          const int col = 32 * c + jx;
-          if (col < NV) acc[col] += (double)__uint_as_float(v[jx]);
-          else if (col < 2 * NV) acc[col - NV] += (double)__uint_as_float(v[jx]);
+        for (int jx = 0; jx < 16; ++jx) {
+          const int col = 16 * c + jx;
+          const float f = __uint_as_float(v[jx]);
+          if (col < NV) {
+            hi[col] = (double)f;
+          } else if (col < 2 * NV) {
+            const int i = col - NV;
+            if (i < 2 * D) {
+              const double x = hi[i] + (double)f;
+              racc[i * kTcTile + row] += (unsigned long long)llrint(x * kFix);
+            } else {  // count: exact integers in both halves
+              const long long nc = llrint(hi[i]) + llrint((double)f);
+              racc[NV * kTcTile + row] += (unsigned long long)nc;
+            }
+          }
         }
       }
     };
     for (int kk = 0; kk < Tg; ++kk) {
       const int jt = 2 * kk + grp;
-      const int s = jt % NST;
+      const int s = jt % NST, sb = jt % C::kNS;
       TcStage<D> st(ring, s);
       long long c0 = clock64();
-      tc::bar_wait(&ms->s_full[grp], kk & 1);
+      tc::bar_wait(&ms->s_full[sb], (jt / C::kNS) & 1);
       tc::fence_after();
       long long c1 = clock64();
       cw[0] += c1 - c0;
 #pragma unroll 1
       for (int c = 0; c < kTcEnt / 32; ++c) {
-        const uint32_t taddr = tb + lane_off + C::kColS + kTcEnt * grp + 32 * c;
+        const uint32_t taddr = tb + lane_off + C::kColS + kTcEnt * sb + 32 * c;
         uint32_t v[32];
         tc::ld32(taddr, v);
         tc::wait_ld();
@@ -883,13 +880,11 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
           mn = __viaddmin_u32(v[jx], 0xFFFFFFFFu, mn);  // min over f > 0 of bits(f) - 1
         }
         if (mn < wm) {  // some pair of this chunk may lie in a band: exact decisions
-          const float* __restrict__ Wv = st.W + 32 * c;
+          // candidates 0 < f <= max band of the chunk (bit trick as for mn); a candidate
+          // outside its own entry's band is still decided exactly below (same answer)
           uint32_t bm = 0u;
 #pragma unroll
-          for (int jx = 0; jx < 32; ++jx) {
-            const float f = __uint_as_float(v[jx]);
-            bm |= (f > 0.f && f <= Wv[jx]) ? (1u << jx) : 0u;
-          }
+          for (int jx = 0; jx < 32; ++jx) bm |= (v[jx] - 1u < wm) ? (1u << jx) : 0u;
           uint32_t fm = 0u;  // band pairs decided inside (single points)
           while (bm) {
             const int jx = __ffs(bm) - 1;
@@ -899,12 +894,12 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
               double s2 = 0.0;
 #pragma unroll
               for (int i = 0; i < D; ++i) {
-                const double t = __dsub_rn((double)st.xc[i * kTcEnt + e], (double)pe[i]);
+                const double t = __dsub_rn((double)a.xs[(int64_t)i * a.n + st.start[e]], (double)pe[i]);
                 s2 = __dadd_rn(s2, __dmul_rn(t, t));
               }
               if (s2 <= a.e2d) fm |= 1u << jx;
             } else {
-              tc_rare<D>(a, pe, e, st, rare, row);
+              tc_rare<D>(a, pe, e, st, racc, row);
             }
           }
 #pragma unroll
@@ -922,7 +917,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
       if (kk >= 1 && ((kk - 1) % kDrain) == kDrain - 1) drain();
       cw[2] += clock64() - c2;
       tc::fence_before();
-      tc::bar_arrive(&ms->p_full[grp]);
+      tc::bar_arrive(&ms->p_full[sb]);
     }
     if (Tg > 0) drain();
     if (a.prof && (tid == 0 || tid == 128)) {
@@ -930,25 +925,19 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
     }
   }
 
-  // ---- epilogue: group 1 hands its sums to group 0 -------------------------------------
-  __syncthreads();  // all MMAs drained; the ring is free
-  double* xch = reinterpret_cast<double*>(ring);
-  if (is_cls && grp == 1) {
-#pragma unroll
-    for (int i = 0; i < NV; ++i) xch[i * kTcTile + row] = acc[i];
-  }
-  __syncthreads();
+  // ---- epilogue (group 0 rows): Eq.5 in fp64 from the exact fixed-point sums -------------
+  __syncthreads();  // all MMAs drained
   if (is_cls && grp == 0 && valid) {
-    const double Nt = acc[2 * D] + xch[2 * D * kTcTile + row];  // tensor-core count (exact integers)
-    const int64_t Ni = (int64_t)Nt + (int64_t)rare[2 * D * kTcTile + row] + (int64_t)a.full_N[j];
+    const unsigned long long* r0 = rare;
+    const unsigned long long* r1 = rare + (NV + 1) * kTcTile;
+    auto fx = [&](int k) { return (long long)(r0[k * kTcTile + row] + r1[k * kTcTile + row]); };
+    const int64_t Nt = fx(NV);  // tensor-core count
+    const int64_t Ni = Nt + fx(2 * D) + (int64_t)a.full_N[j];
     const double inv = 1.0 / (double)Ni;
 #pragma unroll
     for (int i = 0; i < D; ++i) {
-      const double S = acc[i] + xch[i * kTcTile + row] + Nt * (double)ms->s0[i] +
-                       (double)(long long)rare[i * kTcTile + row] * kInvFix + a.full_S[(int64_t)i * a.n + j];
-      const double Cc = acc[D + i] + xch[(D + i) * kTcTile + row] + Nt * (double)ms->c0[i] +
-                        (double)(long long)rare[(D + i) * kTcTile + row] * kInvFix +
-                        a.full_S[(int64_t)(D + i) * a.n + j];
+      const double S = (double)Nt * (double)ms->s0[i] + (double)fx(i) * kInvFix + a.full_S[(int64_t)i * a.n + j];
+      const double Cc = (double)Nt * (double)ms->c0[i] + (double)fx(D + i) * kInvFix + a.full_S[(int64_t)(D + i) * a.n + j];
       double sx, cx;
       const double x = (double)pe[i];
       sincos(x, &sx, &cx);
@@ -961,7 +950,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
   }
   tc::fence_before();
   __syncthreads();
-  if (wid == 11) {
+  if (wid == kMmaWarp) {
     tc::fence_after();
     tc::tmem_dealloc<512>(tb);
   }
@@ -1009,19 +998,29 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     const size_t psmem = (size_t)kPlanWarps * p.stack_len * 8 * sizeof(int);
     const unsigned pgrid = (unsigned)((owned + kPlanWarps - 1) / kPlanWarps);
     EGG_CUDA(cudaFuncSetAttribute(k_tc_plan<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)psmem));
+    p.t_epad = ws.tc_epad;
     // the range buffer keeps its size across updates (process cache); a first guess of
     // 16 chunks per tile, grown and re-planned when the plan reports more
     EGG_TRY(tc_ranges_reserve(ws, (size_t)owned * 16 * kRangeChunk));
-    int32_t hc[2] = {0, 0};
+    size_t tmp = 0;
+    EGG_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, ws.tc_epad, ws.tc_eoff, (int)owned + 1, ws.stream));
+    if (tmp > ws.cub_bytes) {
+      set_error("cub scratch too small for the tensor-core plan scan");
+      return EGGSYNC_ECUDA;
+    }
+    int32_t hc[3] = {0, 0, 0};
     for (int attempt = 0; attempt < 2; ++attempt) {
       p.ranges = ws.tc_ranges;
       p.rcap = (int64_t)ws.tc_rcap;
       EGG_CUDA(cudaMemsetAsync(ws.tc_ctr, 0, 2 * sizeof(int32_t), ws.stream));
+      EGG_CUDA(cudaMemsetAsync(ws.tc_epad + owned, 0, sizeof(int32_t), ws.stream));
       k_tc_plan<D><<<pgrid, kPlanWarps * 32, psmem, ws.stream>>>(p);
       EGG_CUDA(cudaGetLastError());
+      EGG_CUDA(cub::DeviceScan::ExclusiveSum(ws.cub_tmp, tmp, ws.tc_epad, ws.tc_eoff, (int)owned + 1, ws.stream));
       EGG_CUDA(cudaMemcpyAsync(hc, ws.tc_ctr, 2 * sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
+      EGG_CUDA(cudaMemcpyAsync(hc + 2, ws.tc_eoff + owned, sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
       EGG_CUDA(cudaStreamSynchronize(ws.stream));
-      ws.launches += 1;
+      ws.launches += 3;  // plan + scan (2)
       if (hc[1] || (size_t)(uint32_t)hc[0] <= ws.tc_rcap) break;
       EGG_TRY(tc_ranges_reserve(ws, (size_t)(uint32_t)hc[0]));
     }
@@ -1030,6 +1029,11 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
       return run_update_simt<D>(ws, lo, hi, nbr);
     }
     const int32_t total = hc[0];
+    EGG_TRY(tc_ent_reserve(ws, (size_t)(uint32_t)hc[2] + 1));
+    k_tc_expand<0><<<(unsigned)((owned + 3) / 4), 128, 0, ws.stream>>>(ws.tc_ranges, ws.tc_chunks, ws.tc_nr, ws.tc_ne,
+                                                                    ws.tc_eoff, ws.tc_ent, (int32_t)owned);
+    EGG_CUDA(cudaGetLastError());
+    ws.launches += 1;
 
     TcArgs<D> a;
     a.xs = ws.xs[ws.xcur];
@@ -1041,9 +1045,8 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     a.c_rec = ws.c_rec;
     a.c_lo = ws.c_lo;
     a.c_hi = ws.c_hi;
-    a.ranges = ws.tc_ranges;
-    a.chunks = ws.tc_chunks;
-    a.t_nr = ws.tc_nr;
+    a.ent = ws.tc_ent;
+    a.eoff = ws.tc_eoff;
     a.t_ne = ws.tc_ne;
     a.full_S = ws.full_S;
     a.full_N = ws.full_N;
@@ -1092,7 +1095,7 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
       fprintf(stderr, "[tc] n=%lld cells=%d owned_tiles=%lld ranges=%d entries=%lld entry_tiles=%lld max_entries=%lld pairs=%lld\n",
               (long long)ws.n, ws.n_cells, (long long)owned, total, ent, tiles, mx, tiles * kTcEnt * kTcTile);
     }
-    ws.launches += 2;
+    ws.launches += 1;
     return EGGSYNC_OK;
   }
 }
