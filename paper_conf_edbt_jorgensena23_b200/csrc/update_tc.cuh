@@ -982,8 +982,12 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     p.hi = hi;
     p.nc = ws.n_cells;
     p.stack_len = ws.k.keybits + 4;
-    p.bucket = 64;
-    if (const char* e = getenv("EGGSYNC_TC_BUCKET")) p.bucket = atoi(e);
+    // subtrees of <= bucket cells seen partially by the tile become entry ranges: large
+    // while cells are mostly singletons (the tensor cores classify cheaply, the tree walk
+    // does not), smaller once they hold many points each (measured sweep, C3 / C4-d10)
+    const bool singletons = 2 * (int64_t)ws.n_cells > ws.n;
+    p.bucket = singletons ? 512 : 128;
+    if (const char* e = getenv(singletons ? "EGGSYNC_TC_BUCKET_S" : "EGGSYNC_TC_BUCKET")) p.bucket = atoi(e);
     p.ntiles = (int32_t)owned;
     p.stride = ws.own_stride;
     p.offset = ws.own_offset;
