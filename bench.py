@@ -132,8 +132,8 @@ def work_flops(w, d):
     return 2 * d * w["cls"] + 2 * d * w["acc"] + 3 * d * w["scan"] + 6 * d * w["node"]
 
 
-def traffic_from_profiles():
-    p = os.path.join(ROOT, "profiles", "ncu_update_traffic.json")
+def traffic_from_profiles(name="ncu_update_traffic.json"):
+    p = os.path.join(ROOT, "profiles", name)
     try:
         return json.load(open(p)).get("bytes_per_launch")
     except Exception:
@@ -187,10 +187,12 @@ def run_ours(args):
         flush.zero_()
         it, ok, lab = one_step()
     assert ok, "clustering did not converge"
-    # instrumented pass (untimed): algorithmic work of the update launches
+    # instrumented pass (untimed): algorithmic work of the update launches (SIMT kernel
+    # counters; the tensor-core kernel's work is counted from its plan, below)
     ctx.work(enable=1)
     one_step()
     work = ctx.work(enable=0)
+    ctx.tc_work(enable=1)  # time every tensor-core update launch (CUDA events on the library stream)
     # timed region
     hooks = Hooks()
     step_ms = []
@@ -212,6 +214,7 @@ def run_ours(args):
         dist.barrier()
     torch.cuda.synchronize()
     launches = ctx.launches() - launches0
+    tcw = ctx.tc_work(enable=0)
     upd_ms = [a.elapsed_time(b) for a, b in hooks.ev]
     ms = statistics.mean(step_ms)
     if world > 1:
@@ -223,14 +226,34 @@ def run_ours(args):
     iters = it
     value = n * iters / (ms / 1e3)
 
-    # roofline of the dominant kernel (k_update): FP32 pipe
-    flops_per_launch = work_flops(work, d) / iters  # per launch on this rank (its range share)
-    achieved = flops_per_launch / (upd_avg / 1e3) / 1e12
     peaks = load_peaks()
     clk_s = clk.summary()
     fmax = (peaks or {}).get("sm_max_mhz") or clk_s["sm_max_mhz"] or 1965.0
-    peak = 2 * FP32_LANES * SM_COUNT * fmax * 1e6 / 1e12
     upd_share = sum(upd_ms) / sum(step_ms)
+    if tcw["launches"] > 0:
+        # roofline of the dominant kernel, k_update_tc: tf32 tensor cores.  achieved =
+        # algorithmic tensor-core FLOPs per launch (2*pairs*((3d+2)+2(2d+1)), counted from
+        # the plan) / the kernel's own event time; peak = measured sustained bf16 x 1.1/2.25
+        tc_ns = tcw["ns"] / tcw["launches"]
+        flops_per_launch = tcw["flops"] / tcw["launches"]
+        achieved = flops_per_launch / (tc_ns * 1e-9) / 1e12
+        bf16 = (peaks or {}).get("bf16_tflops_sustained")
+        peak = (bf16 if bf16 else 1590.0) * 1.1 / 2.25
+        roof = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+                "traffic": traffic_from_profiles("ncu_update_tc_traffic.json"),
+                "kernel": "k_update_tc (A6 EGG-update on tcgen05, tf32)",
+                "kernel_ms_per_launch": tc_ns / 1e6, "launches_per_step": tcw["launches"] / args.steps,
+                "pairs_per_step": tcw["pairs"] / args.steps,
+                "peak_basis": ("tf32 dense = MEASURED_PEAKS bf16_tflops_sustained x 1.1/2.25 (B200_PROFILING.md nominal ratio)"
+                               if bf16 else "tf32 dense = fallback 1.59 PF bf16 x 1.1/2.25")}
+    else:
+        # roofline of the dominant kernel (SIMT k_update): FP32 pipe
+        flops_per_launch = work_flops(work, d) / iters  # per launch on this rank (its range share)
+        achieved = flops_per_launch / (upd_avg / 1e3) / 1e12
+        peak = 2 * FP32_LANES * SM_COUNT * fmax * 1e6 / 1e12
+        roof = {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+                "traffic": traffic_from_profiles(), "kernel": "k_update (A6 EGG-update)",
+                "peak_basis": f"FP32 FMA pipe 2*128 lanes*148 SMs*{fmax:.0f} MHz (sm_max_mhz, MEASURED_PEAKS.json)"}
 
     # end-to-end through the C ABI with pinned host buffers (rank 0 at N=1 only)
     e2e = None
@@ -270,10 +293,7 @@ def run_ours(args):
                    "l2": "flushed between steps (256 MiB write); inputs resident in HBM",
                    "update_share_of_step": upd_share, "update_ms_per_launch": upd_avg,
                    "launches_per_step": launches / args.steps, "work_counters": work},
-        "roofline": {"bound": "alu", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
-                     "frac": achieved / peak, "traffic": traffic_from_profiles(),
-                     "kernel": "k_update (A6 EGG-update)",
-                     "peak_basis": f"FP32 FMA pipe 2*128 lanes*148 SMs*{fmax:.0f} MHz (sm_max_mhz, MEASURED_PEAKS.json)"},
+        "roofline": roof,
         "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk_s,
     }
     print(json.dumps(line), flush=True)

@@ -206,6 +206,18 @@ void *eggsync_ctx_stream(eggsync_ctx *ctx);
  * pairs, [6] full-subtree uses, [7] staged cells.  Synchronises. */
 int eggsync_ctx_work(eggsync_ctx *ctx, int32_t enable, int64_t *totals_out);
 
+/* Work and time of the tensor-core update kernel (the A6 path taken when d <= 12;
+ * DESIGN.md §6), for its roofline.  enable = 1: reset and time every subsequent
+ * tensor-core update launch with CUDA events on the context stream; 0: stop timing;
+ * -1: leave as is.  out (host, 5 int64, may be NULL) receives the totals since the
+ * last reset, before the enable takes effect: [0] tensor-core update launches,
+ * [1] (point, entry) pairs (128 points x the tile's entries, padding excluded),
+ * [2] pairs including the padding of the last entry tile, [3] algorithmic
+ * tensor-core FLOPs 2*pairs*((3d+2) + 2(2d+1)), [4] summed kernel time in ns
+ * (k_update_tc only; the plan pass is not included).  Synchronises on the last
+ * timed launch.  Returns EGGSYNC_EINVAL for a NULL ctx. */
+int eggsync_ctx_tc_work(eggsync_ctx *ctx, int32_t enable, int64_t *out);
+
 /* Number of kernel launches this context has issued (CUB's internal launches
  * counted per pass). */
 int64_t eggsync_ctx_launches(eggsync_ctx *ctx);

@@ -336,6 +336,12 @@ void Workspace::release() {
   tc_rcap = 0;
   tc_ent = nullptr;
   tc_ecap = 0;
+  for (auto& e : tc_ev)
+    if (e) {
+      cudaEventDestroy(e);
+      e = nullptr;
+    }
+  tc_pending = false;
   arena = nullptr;
   h_flags = nullptr;
   if (own_stream && stream) cudaStreamDestroy(stream);
@@ -840,6 +846,37 @@ int eggsync_ctx_work(eggsync_ctx* ctx, int32_t enable, int64_t* totals_out) {
 }
 
 int64_t eggsync_ctx_launches(eggsync_ctx* ctx) { return ctx ? ctx->ws.launches : -1; }
+
+namespace egg {
+int Workspace::tc_flush() {
+  if (!tc_pending) return EGGSYNC_OK;
+  EGG_CUDA(cudaEventSynchronize(tc_ev[1]));
+  float ms = 0.f;
+  EGG_CUDA(cudaEventElapsedTime(&ms, tc_ev[0], tc_ev[1]));
+  tc_acc[4] += (long long)((double)ms * 1e6);
+  tc_pending = false;
+  return EGGSYNC_OK;
+}
+}  // namespace egg
+
+int eggsync_ctx_tc_work(eggsync_ctx* ctx, int32_t enable, int64_t* out) {
+  if (!ctx) return EGGSYNC_EINVAL;
+  Workspace& ws = ctx->ws;
+  EGG_TRY(ws.tc_flush());
+  if (out)
+    for (int k = 0; k < 5; ++k) out[k] = ws.tc_acc[k];
+  if (enable == 1) {
+    if (!ws.tc_ev[0]) {
+      EGG_CUDA(cudaEventCreate(&ws.tc_ev[0]));
+      EGG_CUDA(cudaEventCreate(&ws.tc_ev[1]));
+    }
+    for (int k = 0; k < 5; ++k) ws.tc_acc[k] = 0;
+    ws.tc_timing = true;
+  } else if (enable == 0) {
+    ws.tc_timing = false;
+  }
+  return EGGSYNC_OK;
+}
 
 int eggsync_ctx_update_owned(eggsync_ctx* ctx, int32_t rank, int32_t ranks) {
   if (!ctx || ranks < 1 || rank < 0 || rank >= ranks) return EGGSYNC_EINVAL;

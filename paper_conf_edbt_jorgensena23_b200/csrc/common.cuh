@@ -230,7 +230,13 @@ struct Workspace {
   int2* tc_ranges = nullptr;    // (first unit, count), grown on demand (process cache)
   size_t tc_rcap = 0;
   int tc_used = 0;              // 1 when the last update ran on the tensor cores
-  long long tc_pairs = 0;       // (point, entry) pairs classified by the last tensor-core update
+  // tensor-core work accounting (eggsync_ctx_tc_work): since the last reset
+  bool tc_timing = false;
+  long long tc_acc[5] = {0, 0, 0, 0, 0};  // launches, pairs (unpadded), pairs (padded), alg FLOPs, kernel ns
+  long long tc_pend_alg = 0;              // FLOPs of the launch whose events are pending
+  bool tc_pending = false;
+  cudaEvent_t tc_ev[2] = {nullptr, nullptr};
+  int tc_flush();                         // fold a pending launch's event time into tc_acc
 
   int alloc(int64_t n, int d, float eps, int device, cudaStream_t stream);
   void release();

@@ -114,7 +114,7 @@ struct PlanArgs {
   int32_t* t_ne;              // [ntiles] entries per tile
   int32_t* t_epad;            // [ntiles] entries padded to whole entry tiles
   int32_t* chunks;            // [ntiles][kChunkMax] first slot of each chunk
-  int32_t* ctr;               // [0] slots allocated, [1] chunk-table overflow
+  int32_t* ctr;               // [0] slots allocated, [1] chunk-table overflow, [2..3] entries (u64)
   int64_t rcap;               // capacity of ranges
   int2* ranges;               // (first cell, count)
   double* full_S;             // [2D][n]
@@ -299,6 +299,7 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
   if (lane == 0) {
     a.t_nr[tile] = nr;
     a.t_ne[tile] = ne;
+    atomicAdd(reinterpret_cast<unsigned long long*>(a.ctr + 2), (unsigned long long)ne);  // unpadded entries
     a.t_epad[tile] = (ne + kTcEnt - 1) / kTcEnt * kTcEnt;
   }
 #pragma unroll
@@ -969,7 +970,6 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     const int64_t owned =
         ntot > ws.own_offset ? (ntot - ws.own_offset + ws.own_stride - 1) / ws.own_stride : 0;
     ws.tc_used = 1;
-    ws.tc_pairs = 0;
     if (owned == 0) return EGGSYNC_OK;
     PlanArgs<D> p;
     p.xs = ws.xs[ws.xcur];
@@ -1012,17 +1012,17 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
       set_error("cub scratch too small for the tensor-core plan scan");
       return EGGSYNC_ECUDA;
     }
-    int32_t hc[3] = {0, 0, 0};
+    int32_t hc[5] = {0, 0, 0, 0, 0};  // ctr[0..3], padded entries
     for (int attempt = 0; attempt < 2; ++attempt) {
       p.ranges = ws.tc_ranges;
       p.rcap = (int64_t)ws.tc_rcap;
-      EGG_CUDA(cudaMemsetAsync(ws.tc_ctr, 0, 2 * sizeof(int32_t), ws.stream));
+      EGG_CUDA(cudaMemsetAsync(ws.tc_ctr, 0, 4 * sizeof(int32_t), ws.stream));
       EGG_CUDA(cudaMemsetAsync(ws.tc_epad + owned, 0, sizeof(int32_t), ws.stream));
       k_tc_plan<D><<<pgrid, kPlanWarps * 32, psmem, ws.stream>>>(p);
       EGG_CUDA(cudaGetLastError());
       EGG_CUDA(cub::DeviceScan::ExclusiveSum(ws.cub_tmp, tmp, ws.tc_epad, ws.tc_eoff, (int)owned + 1, ws.stream));
-      EGG_CUDA(cudaMemcpyAsync(hc, ws.tc_ctr, 2 * sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
-      EGG_CUDA(cudaMemcpyAsync(hc + 2, ws.tc_eoff + owned, sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
+      EGG_CUDA(cudaMemcpyAsync(hc, ws.tc_ctr, 4 * sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
+      EGG_CUDA(cudaMemcpyAsync(hc + 4, ws.tc_eoff + owned, sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
       EGG_CUDA(cudaStreamSynchronize(ws.stream));
       ws.launches += 3;  // plan + scan (2)
       if (hc[1] || (size_t)(uint32_t)hc[0] <= ws.tc_rcap) break;
@@ -1032,8 +1032,7 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
       ws.tc_used = 0;
       return run_update_simt<D>(ws, lo, hi, nbr);
     }
-    const int32_t total = hc[0];
-    EGG_TRY(tc_ent_reserve(ws, (size_t)(uint32_t)hc[2] + 1));
+    EGG_TRY(tc_ent_reserve(ws, (size_t)(uint32_t)hc[4] + 1));
     k_tc_expand<0><<<(unsigned)((owned + 3) / 4), 128, 0, ws.stream>>>(ws.tc_ranges, ws.tc_chunks, ws.tc_nr, ws.tc_ne,
                                                                     ws.tc_eoff, ws.tc_ent, (int32_t)owned);
     EGG_CUDA(cudaGetLastError());
@@ -1075,8 +1074,26 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
       a.prof = prof;
     }
     EGG_CUDA(cudaFuncSetAttribute(k_update_tc<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::kSmem));
+    if (ws.tc_timing) {
+      EGG_TRY(ws.tc_flush());
+      unsigned long long ent_u = 0;
+      memcpy(&ent_u, hc + 2, sizeof(ent_u));
+      const long long pairs = (long long)ent_u * kTcTile, padded = (long long)(uint32_t)hc[4] * kTcTile;
+      ws.tc_acc[0] += 1;
+      ws.tc_acc[1] += pairs;
+      ws.tc_acc[2] += padded;
+      // algorithmic tensor-core FLOPs: GEMM1 over the 3D+2 operand columns, GEMM2 over the
+      // 2(2D+1) value columns (hi/lo split), per (point, entry) pair
+      ws.tc_pend_alg = 2LL * pairs * ((3 * D + 2) + 2 * (2 * D + 1));
+      ws.tc_acc[3] += ws.tc_pend_alg;
+      EGG_CUDA(cudaEventRecord(ws.tc_ev[0], ws.stream));
+    }
     k_update_tc<D><<<(unsigned)owned, kTcThreads, C::kSmem, ws.stream>>>(a);
     EGG_CUDA(cudaGetLastError());
+    if (ws.tc_timing) {
+      EGG_CUDA(cudaEventRecord(ws.tc_ev[1], ws.stream));
+      ws.tc_pending = true;
+    }
     if (a.prof) {
       unsigned long long h[16];
       EGG_CUDA(cudaMemcpyAsync(h, prof, sizeof(h), cudaMemcpyDeviceToHost, ws.stream));
@@ -1097,7 +1114,7 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
         mx = v > mx ? v : mx;
       }
       fprintf(stderr, "[tc] n=%lld cells=%d owned_tiles=%lld ranges=%d entries=%lld entry_tiles=%lld max_entries=%lld pairs=%lld\n",
-              (long long)ws.n, ws.n_cells, (long long)owned, total, ent, tiles, mx, tiles * kTcEnt * kTcTile);
+              (long long)ws.n, ws.n_cells, (long long)owned, hc[0], ent, tiles, mx, tiles * kTcEnt * kTcTile);
     }
     ws.launches += 1;
     return EGGSYNC_OK;

@@ -25,7 +25,7 @@ SYMBOLS = [
     "eggsync_ctx_load", "eggsync_ctx_build", "eggsync_ctx_update", "eggsync_ctx_second_term",
     "eggsync_ctx_flags", "eggsync_ctx_cur_coords", "eggsync_ctx_next_coords", "eggsync_ctx_pack",
     "eggsync_ctx_unpack", "eggsync_ctx_advance", "eggsync_ctx_labels", "eggsync_ctx_coords",
-    "eggsync_ctx_run", "eggsync_ctx_stream", "eggsync_ctx_work", "eggsync_ctx_launches",
+    "eggsync_ctx_run", "eggsync_ctx_stream", "eggsync_ctx_work", "eggsync_ctx_tc_work", "eggsync_ctx_launches",
     "eggsync_release_cache", "eggsync_ctx_update_owned", "eggsync_ctx_owned_count", "eggsync_ctx_pack_owned",
     "eggsync_ctx_unpack_owned",
 ]
@@ -92,6 +92,7 @@ def lib():
             "eggsync_ctx_run": ([vp, i32, vp], ctypes.c_int),
             "eggsync_ctx_stream": ([vp], vp),
             "eggsync_ctx_work": ([vp, i32, vp], ctypes.c_int),
+            "eggsync_ctx_tc_work": ([vp, i32, vp], ctypes.c_int),
             "eggsync_ctx_launches": ([vp], ctypes.c_int64),
             "eggsync_release_cache": ([], None),
             "eggsync_ctx_update_owned": ([vp, i32, i32], ctypes.c_int),
@@ -310,6 +311,14 @@ class Context:
         out = np.zeros(8, np.int64)
         _check(lib().eggsync_ctx_work(self.h, enable, out.ctypes.data_as(ctypes.c_void_p)))
         return dict(zip(self.WORK_KEYS, out.tolist()))
+
+    TC_KEYS = ("launches", "pairs", "pairs_padded", "flops", "ns")
+
+    def tc_work(self, enable: int = -1):
+        """Tensor-core update work / kernel time (dict), then set timing on (1) / off (0) / unchanged (-1)."""
+        out = np.zeros(5, np.int64)
+        _check(lib().eggsync_ctx_tc_work(self.h, enable, out.ctypes.data_as(ctypes.c_void_p)))
+        return dict(zip(self.TC_KEYS, out.tolist()))
 
     def launches(self) -> int:
         return int(lib().eggsync_ctx_launches(self.h))

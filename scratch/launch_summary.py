@@ -7,7 +7,7 @@ agg = defaultdict(float); cnt = defaultdict(int); seq = []
 for x in d:
     if x['Metric Name'] != 'gpu__time_duration.sum': continue
     v = float(x['Metric Value'].replace(',', ''))
-    v *= {'nsecond': 1, 'usecond': 1e3, 'msecond': 1e6}.get(x['Metric Unit'], 1)
+    v *= {'nsecond': 1, 'ns': 1, 'usecond': 1e3, 'us': 1e3, 'msecond': 1e6, 'ms': 1e6}.get(x['Metric Unit'], 1)
     k = x['Kernel Name'][:60]
     agg[k] += v; cnt[k] += 1; seq.append((k, v))
 tot = sum(agg.values())
