@@ -278,6 +278,9 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
       {(void**)&tc_ctr, sizeof(int32_t) * 4},
       {(void**)&tc_epad, sizeof(int32_t) * (n / 128 + 2)},
       {(void**)&tc_eoff, sizeof(int32_t) * (n / 128 + 2)},
+      {(void**)&tc_pv, sizeof(int32_t) * (n / 128 + 2)},
+      {(void**)&tc_pk, sizeof(int32_t) * (n / 128 + 2)},
+      {(void**)&tc_perm, sizeof(int32_t) * (n / 128 + 2)},
       {(void**)&co_start, sizeof(int32_t) * (cap + 1)},
       {(void**)&co_cnt, sizeof(int32_t) * cap},
       {(void**)&co_lo, sizeof(uint32_t) * d * cap},

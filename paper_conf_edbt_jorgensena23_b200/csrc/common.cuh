@@ -226,6 +226,9 @@ struct Workspace {
   int32_t* tc_epad = nullptr;   // [tiles+1] entries per tile padded to whole entry tiles
   int32_t* tc_eoff = nullptr;   // [tiles+1] first entry of each tile in tc_ent (exclusive scan)
   int32_t* tc_ent = nullptr;    // unit (cell) of every entry slot, -1 = padding (grown on demand)
+  int32_t* tc_pv = nullptr;     // [tiles] tile index (sort values)
+  int32_t* tc_pk = nullptr;     // [tiles] entries, sorted descending (sort keys out)
+  int32_t* tc_perm = nullptr;   // [tiles] launch order of the point tiles: most entries first
   size_t tc_ecap = 0;
   int2* tc_ranges = nullptr;    // (first unit, count), grown on demand (process cache)
   size_t tc_rcap = 0;

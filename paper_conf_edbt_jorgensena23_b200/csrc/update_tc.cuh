@@ -113,6 +113,7 @@ struct PlanArgs {
   int32_t* t_nr;              // [ntiles] ranges per tile
   int32_t* t_ne;              // [ntiles] entries per tile
   int32_t* t_epad;            // [ntiles] entries padded to whole entry tiles
+  int32_t* t_pv;              // [ntiles] tile index (values of the launch-order sort)
   int32_t* chunks;            // [ntiles][kChunkMax] first slot of each chunk
   int32_t* ctr;               // [0] slots allocated, [1] chunk-table overflow, [2..3] entries (u64)
   int64_t rcap;               // capacity of ranges
@@ -301,6 +302,7 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
     a.t_ne[tile] = ne;
     atomicAdd(reinterpret_cast<unsigned long long*>(a.ctr + 2), (unsigned long long)ne);  // unpadded entries
     a.t_epad[tile] = (ne + kTcEnt - 1) / kTcEnt * kTcEnt;
+    a.t_pv[tile] = (int32_t)tile;
   }
 #pragma unroll
   for (int k = 0; k < kP; ++k) {
@@ -368,6 +370,7 @@ struct TcArgs {
   const uint32_t* __restrict__ c_hi;
   const int32_t* __restrict__ ent;   // unit of every entry slot (-1 = padding)
   const int32_t* __restrict__ eoff;  // [ntiles] first slot of each point tile
+  const int32_t* __restrict__ perm;  // [ntiles] launch order
   const int32_t* __restrict__ t_ne;
   const double* __restrict__ full_S;
   const int32_t* __restrict__ full_N;
@@ -598,7 +601,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
   TcMisc* ms = reinterpret_cast<TcMisc*>(tsm + C::kRingBytes + C::kRawBytes + C::kRareBytes);
 
   const int tid = threadIdx.x, wid = tid >> 5, lane = tid & 31;
-  const int64_t tile = blockIdx.x;
+  const int64_t tile = a.perm[blockIdx.x];  // heaviest point tiles first (shorter tail)
   const int64_t base = tc_tile_base(a.lo, tile, a.stride, a.offset);
   const int32_t ne = a.t_ne[tile];
   const int T = (ne + kTcEnt - 1) / kTcEnt;  // entry tiles (the slot list is padded to T * kTcEnt)
@@ -1003,6 +1006,7 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     const unsigned pgrid = (unsigned)((owned + kPlanWarps - 1) / kPlanWarps);
     EGG_CUDA(cudaFuncSetAttribute(k_tc_plan<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)psmem));
     p.t_epad = ws.tc_epad;
+    p.t_pv = ws.tc_pv;
     // the range buffer keeps its size across updates (process cache); a first guess of
     // 16 chunks per tile, grown and re-planned when the plan reports more
     EGG_TRY(tc_ranges_reserve(ws, (size_t)owned * 16 * kRangeChunk));
@@ -1037,6 +1041,19 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
                                                                     ws.tc_eoff, ws.tc_ent, (int32_t)owned);
     EGG_CUDA(cudaGetLastError());
     ws.launches += 1;
+    // launch order: point tiles by descending entry count (longest-processing-time first)
+    {
+      size_t stmp = 0;
+      EGG_CUDA(cub::DeviceRadixSort::SortPairsDescending(nullptr, stmp, ws.tc_ne, ws.tc_pk, ws.tc_pv, ws.tc_perm,
+                                                         (int)owned, 0, 32, ws.stream));
+      if (stmp > ws.cub_bytes) {
+        set_error("cub scratch too small for the tensor-core tile order");
+        return EGGSYNC_ECUDA;
+      }
+      EGG_CUDA(cub::DeviceRadixSort::SortPairsDescending(ws.cub_tmp, stmp, ws.tc_ne, ws.tc_pk, ws.tc_pv, ws.tc_perm,
+                                                         (int)owned, 0, 32, ws.stream));
+      ws.launches += 4;
+    }
 
     TcArgs<D> a;
     a.xs = ws.xs[ws.xcur];
@@ -1050,6 +1067,7 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     a.c_hi = ws.c_hi;
     a.ent = ws.tc_ent;
     a.eoff = ws.tc_eoff;
+    a.perm = ws.tc_perm;
     a.t_ne = ws.tc_ne;
     a.full_S = ws.full_S;
     a.full_N = ws.full_N;
