@@ -275,7 +275,7 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
       {(void**)&tc_nr, sizeof(int32_t) * (n / 128 + 2)},
       {(void**)&tc_ne, sizeof(int32_t) * (n / 128 + 2)},
       {(void**)&tc_chunks, d <= 16 ? sizeof(int32_t) * (n / 128 + 2) * kChunkMax : 0},
-      {(void**)&tc_ctr, sizeof(int32_t) * 4},
+      {(void**)&tc_ctr, sizeof(int32_t) * 8},
       {(void**)&tc_epad, sizeof(int32_t) * (n / 128 + 2)},
       {(void**)&tc_eoff, sizeof(int32_t) * (n / 128 + 2)},
       {(void**)&tc_pv, sizeof(int32_t) * (n / 128 + 2)},

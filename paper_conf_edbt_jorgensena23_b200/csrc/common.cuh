@@ -222,7 +222,7 @@ struct Workspace {
   int32_t* tc_nr = nullptr;     // [tiles+1] ranges per point tile
   int32_t* tc_ne = nullptr;     // [tiles+1] entries per point tile
   int32_t* tc_chunks = nullptr; // [tiles][kChunkMax] first range of each chunk of a tile's range list
-  int32_t* tc_ctr = nullptr;    // [4] ranges allocated, chunk-table overflow
+  int32_t* tc_ctr = nullptr;    // [8] ranges allocated, chunk-table overflow, entries (u64), points in entries (u64)
   int32_t* tc_epad = nullptr;   // [tiles+1] entries per tile padded to whole entry tiles
   int32_t* tc_eoff = nullptr;   // [tiles+1] first entry of each tile in tc_ent (exclusive scan)
   int32_t* tc_ent = nullptr;    // unit (cell) of every entry slot, -1 = padding (grown on demand)

@@ -107,6 +107,7 @@ struct PlanArgs {
   const float* __restrict__ t_box;
   const float* __restrict__ t_sum;
   const int32_t* __restrict__ t_cnt;
+  const int32_t* __restrict__ c_cnt;  // points per unit (cell)
   int64_t n, lo, hi;
   int32_t nc, stack_len, bucket, ntiles, stride, offset;
   float e;
@@ -115,7 +116,7 @@ struct PlanArgs {
   int32_t* t_epad;            // [ntiles] entries padded to whole entry tiles
   int32_t* t_pv;              // [ntiles] tile index (values of the launch-order sort)
   int32_t* chunks;            // [ntiles][kChunkMax] first slot of each chunk
-  int32_t* ctr;               // [0] slots allocated, [1] chunk-table overflow, [2..3] entries (u64)
+  int32_t* ctr;               // [0] slots allocated, [1] chunk-table overflow, [2..3] entries (u64), [4..5] their points (u64)
   int64_t rcap;               // capacity of ranges
   int2* ranges;               // (first cell, count)
   double* full_S;             // [2D][n]
@@ -187,10 +188,12 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
   bool touched[kP] = {false, false, false, false};  // full_S of the point initialised
   int N[kP] = {0, 0, 0, 0};
   int32_t nr = 0, ne = 0;
+  long long npts = 0;  // points in the tile's entries (= ne while the cells are singletons)
   int32_t cbase = 0;  // first slot of the current chunk (warp-uniform)
   int32_t* __restrict__ tch = a.chunks + tile * kChunkMax;
   // append a range (warp-uniform call)
-  auto push = [&](int32_t first, int32_t cnt) {
+  auto push = [&](int32_t first, int32_t cnt, int32_t pts) {
+    npts += pts;
     const int32_t slot = nr % kRangeChunk;
     if (slot == 0) {
       int32_t b = 0;
@@ -223,7 +226,7 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
     for (int k = 0; k < kP; ++k) m[k] = (uint32_t)stk[sp * 8 + 1 + k];
     __syncwarp();
     if (node & (int)kLeafBit) {  // a single cell: always an entry
-      push(node & 0x7fffffff, 1);
+      push(node & 0x7fffffff, 1, a.c_cnt[node & 0x7fffffff]);
       continue;
     }
     const float* __restrict__ bx = a.t_box + (int64_t)node * BS;
@@ -278,7 +281,7 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
     const int4 meta = a.t_meta[node];
     const int ncell = meta.y - meta.x + 1;
     if (ncell <= a.bucket) {
-      push(meta.x, ncell);
+      push(meta.x, ncell, a.t_cnt[node]);
       continue;
     }
     if (sp + 2 > a.stack_len) {
@@ -301,6 +304,7 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
     a.t_nr[tile] = nr;
     a.t_ne[tile] = ne;
     atomicAdd(reinterpret_cast<unsigned long long*>(a.ctr + 2), (unsigned long long)ne);  // unpadded entries
+    atomicAdd(reinterpret_cast<unsigned long long*>(a.ctr + 4), (unsigned long long)npts);
     a.t_epad[tile] = (ne + kTcEnt - 1) / kTcEnt * kTcEnt;
     a.t_pv[tile] = (int32_t)tile;
   }
@@ -980,6 +984,7 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     p.t_box = ws.t_box;
     p.t_sum = ws.t_sum;
     p.t_cnt = ws.t_cnt;
+    p.c_cnt = ws.c_cnt;
     p.n = ws.n;
     p.lo = lo;
     p.hi = hi;
@@ -1016,17 +1021,17 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
       set_error("cub scratch too small for the tensor-core plan scan");
       return EGGSYNC_ECUDA;
     }
-    int32_t hc[5] = {0, 0, 0, 0, 0};  // ctr[0..3], padded entries
+    int32_t hc[7] = {0, 0, 0, 0, 0, 0, 0};  // ctr[0..5], padded entries
     for (int attempt = 0; attempt < 2; ++attempt) {
       p.ranges = ws.tc_ranges;
       p.rcap = (int64_t)ws.tc_rcap;
-      EGG_CUDA(cudaMemsetAsync(ws.tc_ctr, 0, 4 * sizeof(int32_t), ws.stream));
+      EGG_CUDA(cudaMemsetAsync(ws.tc_ctr, 0, 6 * sizeof(int32_t), ws.stream));
       EGG_CUDA(cudaMemsetAsync(ws.tc_epad + owned, 0, sizeof(int32_t), ws.stream));
       k_tc_plan<D><<<pgrid, kPlanWarps * 32, psmem, ws.stream>>>(p);
       EGG_CUDA(cudaGetLastError());
       EGG_CUDA(cub::DeviceScan::ExclusiveSum(ws.cub_tmp, tmp, ws.tc_epad, ws.tc_eoff, (int)owned + 1, ws.stream));
-      EGG_CUDA(cudaMemcpyAsync(hc, ws.tc_ctr, 4 * sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
-      EGG_CUDA(cudaMemcpyAsync(hc + 4, ws.tc_eoff + owned, sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
+      EGG_CUDA(cudaMemcpyAsync(hc, ws.tc_ctr, 6 * sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
+      EGG_CUDA(cudaMemcpyAsync(hc + 6, ws.tc_eoff + owned, sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
       EGG_CUDA(cudaStreamSynchronize(ws.stream));
       ws.launches += 3;  // plan + scan (2)
       if (hc[1] || (size_t)(uint32_t)hc[0] <= ws.tc_rcap) break;
@@ -1036,7 +1041,22 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
       ws.tc_used = 0;
       return run_update_simt<D>(ws, lo, hi, nbr);
     }
-    EGG_TRY(tc_ent_reserve(ws, (size_t)(uint32_t)hc[4] + 1));
+    unsigned long long ent_u = 0, pts_u = 0;
+    memcpy(&ent_u, hc + 2, sizeof(ent_u));
+    memcpy(&pts_u, hc + 4, sizeof(pts_u));
+    const double occ = ent_u ? (double)pts_u / (double)ent_u : 1.0;
+    if (getenv("EGGSYNC_TC_DEBUG"))
+      fprintf(stderr, "[tc-plan] entries=%llu points_in_entries=%llu ratio=%.3f\n", ent_u, pts_u, occ);
+    // Entries holding a few points each on average (partly collapsed clusters) put many
+    // multi-point cells in the classifiers' exact band, where one lane scans a cell's points
+    // alone; the warp-cooperative SIMT kernel is faster there (measured: C4-d10 iterations
+    // 5-7, C4-d5 / C2 late iterations).  Singletons (occ ~ 1) and fully collapsed clusters
+    // (occ >= 50: whole-cell summaries) stay on the tensor cores.
+    if (occ > 1.1 && occ < 50.0) {
+      ws.tc_used = 0;
+      return run_update_simt<D>(ws, lo, hi, nbr);
+    }
+    EGG_TRY(tc_ent_reserve(ws, (size_t)(uint32_t)hc[6] + 1));
     k_tc_expand<0><<<(unsigned)((owned + 3) / 4), 128, 0, ws.stream>>>(ws.tc_ranges, ws.tc_chunks, ws.tc_nr, ws.tc_ne,
                                                                     ws.tc_eoff, ws.tc_ent, (int32_t)owned);
     EGG_CUDA(cudaGetLastError());
@@ -1094,9 +1114,7 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     EGG_CUDA(cudaFuncSetAttribute(k_update_tc<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::kSmem));
     if (ws.tc_timing) {
       EGG_TRY(ws.tc_flush());
-      unsigned long long ent_u = 0;
-      memcpy(&ent_u, hc + 2, sizeof(ent_u));
-      const long long pairs = (long long)ent_u * kTcTile, padded = (long long)(uint32_t)hc[4] * kTcTile;
+      const long long pairs = (long long)ent_u * kTcTile, padded = (long long)(uint32_t)hc[6] * kTcTile;
       ws.tc_acc[0] += 1;
       ws.tc_acc[1] += pairs;
       ws.tc_acc[2] += padded;
@@ -1140,13 +1158,16 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
 }
 
 // tensor cores when the dimension fits the TMEM / shared-memory budget and the fp32
-// tensor-core count sums stay exact (n < 2^24); EGGSYNC_TC=0 forces the SIMT kernel
+// tensor-core count sums stay exact (n < 2^24); EGGSYNC_TC=0 forces the SIMT kernel,
+// EGGSYNC_TC=2 the tensor cores also for small cell counts
 inline bool tc_enabled(const Workspace& ws, int d) {
   static const int env = [] {
     const char* e = getenv("EGGSYNC_TC");
     return e ? atoi(e) : 1;
   }();
-  return env != 0 && d <= kTcMaxD && ws.n < (int64_t(1) << 24);
+  // (a few thousand cells: fully collapsed clusters, the plan / sync overhead of the
+  // tensor-core path exceeds the whole SIMT update)
+  return env != 0 && d <= kTcMaxD && ws.n < (int64_t(1) << 24) && (ws.n_cells >= 4096 || env == 2);
 }
 
 template <int D>
