@@ -17,18 +17,23 @@
 //   GEMM2  O[p][:] += P[p][:] . V[:][:]        V_e = (sum sin - cnt sin o, sum cos - cnt cos o, cnt)
 //                                              split hi/lo into tf32 pairs (N = 2(2D+1))
 //
-// with fp32 accumulation in TMEM drained into fp64 registers every kDrain entry tiles.
+// with fp32 accumulation in TMEM drained every kDrain entry tiles into exact 64-bit
+// fixed-point sums (2^-32) per classifier group in shared memory.
 // Entries are the cells of the subtrees that the plan pass (k_tc_plan) could not
 // decide for the whole tile; subtrees entirely inside for every point that still
 // needs them are added per point in the plan pass (full_S / full_N, exact fp64 of
-// the fp32 subtree sums, as in k_update).
+// the fp32 subtree sums, as in k_update).  k_tc_expand turns each tile's ranges into a
+// slot list (one unit per entry, padded to whole entry tiles); tiles are launched
+// heaviest-first.
 //
-// Roles (384 threads, one CTA per point tile, one CTA per SM: it owns all 512 TMEM columns):
-//   warps 0-3  classifier group 0 (TMEM lanes 0..127), even entry tiles
-//   warps 4-7  classifier group 1, odd entry tiles
-//   warps 8-10 producers: expand the tile's ranges into 128 entries per entry tile and write
-//              the GEMM operands (origin-shifted, tf32-split) into a shared-memory ring
-//   warp 11    MMA issue (one elected thread) and TMEM owner
+// Roles (416 threads, one CTA per point tile, one CTA per SM: it owns all 512 TMEM columns):
+//   warps 0-3   classifier group 0 (TMEM lanes 0..127), even entry tiles
+//   warps 4-7   classifier group 1, odd entry tiles
+//   warps 8-11  producers: thread t owns entry slot t; stages the unit record with
+//               cp.async one tile ahead and writes the GEMM operands (origin-shifted,
+//               tf32-split) into a 3-stage shared-memory ring
+//   warp 12     MMA issue (one thread, polling both GEMM conditions) and TMEM owner
+// TMEM: Q (K1 columns) | 3 S/P buffers (GEMM1 runs up to 2 tiles ahead) | O per group.
 #pragma once
 #include <cub/cub.cuh>
 
