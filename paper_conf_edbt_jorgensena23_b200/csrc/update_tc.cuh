@@ -753,13 +753,12 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
         fetch(c_nxt, sb ^ 1);
         c_cur = c_nxt;
         c_nxt = unit_of(jt + 2);
-        cp_async_wait<1>();
-      } else {
-        cp_async_wait<0>();
       }
       long long t1 = clock64();
-      long long t2 = t1;
-      if (jt >= NST) tc::bar_wait(&ms->stage_empty[s], ((jt / NST) - 1) & 1);
+      if (jt >= NST) tc::bar_wait(&ms->stage_empty[s], ((jt / NST) - 1) & 1);  // overlaps the copies
+      long long t2 = clock64();
+      if (jt + 1 < T) cp_async_wait<1>();
+      else cp_async_wait<0>();
       long long t3 = clock64();
       pc[0] += t1 - t0;
       pc[1] += t2 - t1;
@@ -1140,7 +1139,7 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
       EGG_CUDA(cudaMemcpyAsync(h, prof, sizeof(h), cudaMemcpyDeviceToHost, ws.stream));
       EGG_CUDA(cudaStreamSynchronize(ws.stream));
       const double t = (double)(h[4] ? h[4] : 1);
-      fprintf(stderr, "[tc-prof] per entry tile (clk): producer expand %.0f wait_raw %.0f wait_empty %.0f build %.0f | "
+      fprintf(stderr, "[tc-prof] per entry tile (clk): producer fetch %.0f wait_empty %.0f wait_records %.0f build %.0f | "
               "classifier wait_S %.0f classify %.0f drain %.0f\n", h[0] / t, h[1] / t, h[2] / t, h[3] / t,
               2 * h[5] / t, 2 * h[6] / t, 2 * h[7] / t);
     }
