@@ -824,7 +824,10 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
           ++j2;
           did = true;
         }
-        if (!did) __nanosleep(20);
+        if (!did) {  // sleep on the event most likely next: P of the oldest issued GEMM1
+          if (j2 < j1) tc::bar_try(&ms->p_full[j2 % NS], (j2 / NS) & 1, 200);
+          else if (j1 < T) tc::bar_try(&ms->stage_full[j1 % NST], (j1 / NST) & 1, 200);
+        }
       }
     }
     __syncwarp();
