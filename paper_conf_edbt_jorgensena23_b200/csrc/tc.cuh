@@ -32,29 +32,6 @@ __device__ __forceinline__ void bar_wait(uint64_t* b, uint32_t parity) {
       : "memory");
 }
 
-// non-blocking test of a phase (true once the phase with this parity has completed)
-__device__ __forceinline__ bool bar_test(uint64_t* b, uint32_t parity) {
-  uint32_t ok;
-  asm volatile(
-      "{\n .reg .pred p;\n mbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n selp.u32 %0, 1, 0, p;\n}"
-      : "=r"(ok)
-      : "r"(smem_addr(b)), "r"(parity)
-      : "memory");
-  return ok != 0;
-}
-
-// bounded blocking test: suspends the thread until the phase completes or about
-// `hint_ns` elapse (no issue slots spent spinning); true once the phase completed
-__device__ __forceinline__ bool bar_try(uint64_t* b, uint32_t parity, uint32_t hint_ns) {
-  uint32_t ok;
-  asm volatile(
-      "{\n .reg .pred p;\n mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n selp.u32 %0, 1, 0, p;\n}"
-      : "=r"(ok)
-      : "r"(smem_addr(b)), "r"(parity), "r"(hint_ns)
-      : "memory");
-  return ok != 0;
-}
-
 // ---- TMEM allocation (one warp, power-of-two columns >= 32) -----------------
 template <uint32_t kCols>
 __device__ __forceinline__ void tmem_alloc(uint32_t* dst_smem) {

@@ -784,21 +784,21 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
   if (wid == kMmaWarp) {
     // ================================ MMA issue ================================
     // One thread issues, in order (the tensor pipe executes them in order):
-    //   GEMM1(j1)  S[j1 % NS] = Q . B1(j1)^T      once stage j1 is built, and only after
-    //              GEMM2(j1 - NS) (the last reader of that S buffer) was issued
-    //   GEMM2(j2)  O[g] (+)= P . B2(j2)^T         once its classifier group wrote P
-    // polling both conditions, so neither kind waits behind the other.
+    //   GEMM1(jt)        S[jt % NS] = Q . B1(jt)^T      once stage jt is built
+    //   GEMM2(jt-NS+1)   O[g] (+)= P . B2^T             once its classifier group wrote P
+    // so GEMM1 runs NS-1 tiles ahead of the classifiers and GEMM1(jt) follows GEMM2(jt-NS),
+    // the last reader of its S buffer.  Blocking waits (the warp is suspended, it does not
+    // take issue slots from the classifier / producer warps of its sub-partition).
     if (lane == 0) {
       constexpr uint32_t id1 = tc::idesc_tf32(128, kTcEnt, false);
       constexpr uint32_t id2 = tc::idesc_tf32(128, N2, false);
       constexpr int NS = C::kNS;
       const uint32_t ring_s = tc::smem_addr(ring);
       const int T0 = (T + 1) / 2, T1 = T / 2;  // entry tiles of group 0 / 1
-      int j1 = 0, j2 = 0;
-      while (j2 < T) {
-        bool did = false;
-        if (j1 < T && j1 - j2 < NS && tc::bar_test(&ms->stage_full[j1 % NST], (j1 / NST) & 1)) {
-          const int s = j1 % NST, sb = j1 % NS;
+      for (int jt = 0; jt < T + NS - 1; ++jt) {
+        if (jt < T) {
+          const int s = jt % NST, sb = jt % NS;
+          tc::bar_wait(&ms->stage_full[s], (jt / NST) & 1);
           tc::fence_after();
           const uint32_t b1 = ring_s + s * C::kStageBytes;
 #pragma unroll
@@ -806,11 +806,11 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
             tc::mma_ts(tb + C::kColS + kTcEnt * sb, tb + C::kColQ + 8 * k, tc::sdesc(b1 + k * 256, 128, C::SBO1), id1,
                        k > 0);
           tc::mma_commit(&ms->s_full[sb]);
-          ++j1;
-          did = true;
         }
-        if (j2 < j1 && tc::bar_test(&ms->p_full[j2 % NS], (j2 / NS) & 1)) {  // per S buffer: never two phases ahead
-          const int jj = j2, s = jj % NST, sb = jj % NS, g = jj & 1, kk = jj >> 1;
+        const int jj = jt - (NS - 1);
+        if (jj >= 0 && jj < T) {
+          const int s = jj % NST, sb = jj % NS, g = jj & 1, kk = jj >> 1;
+          tc::bar_wait(&ms->p_full[sb], (jj / NS) & 1);  // per S buffer: never two phases ahead
           tc::fence_after();
           const uint32_t b2 = ring_s + s * C::kStageBytes + C::kB1Bytes;
           const uint32_t acc0 = (kk % kDrain) != 0;
@@ -821,12 +821,6 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
           tc::mma_commit(&ms->stage_empty[s]);
           const int Tg = g ? T1 : T0;
           if ((kk % kDrain) == kDrain - 1 || kk == Tg - 1) tc::mma_commit(&ms->o_full[g]);
-          ++j2;
-          did = true;
-        }
-        if (!did) {  // sleep on the event most likely next: P of the oldest issued GEMM1
-          if (j2 < j1) tc::bar_try(&ms->p_full[j2 % NS], (j2 / NS) & 1, 200);
-          else if (j1 < T) tc::bar_try(&ms->stage_full[j1 % NST], (j1 / NST) & 1, 200);
         }
       }
     }
