@@ -1047,13 +1047,19 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     memcpy(&pts_u, hc + 4, sizeof(pts_u));
     const double occ = ent_u ? (double)pts_u / (double)ent_u : 1.0;
     if (getenv("EGGSYNC_TC_DEBUG"))
-      fprintf(stderr, "[tc-plan] entries=%llu points_in_entries=%llu ratio=%.3f\n", ent_u, pts_u, occ);
+      fprintf(stderr, "[tc-plan] entries=%llu points_in_entries=%llu ratio=%.3f slots=%d overflow=%d padded=%d rcap=%zu tiles=%lld\n",
+              ent_u, pts_u, occ, hc[0], hc[1], hc[6], ws.tc_rcap, (long long)owned);
     // Entries holding a few points each on average (partly collapsed clusters) put many
     // multi-point cells in the classifiers' exact band, where one lane scans a cell's points
     // alone; the warp-cooperative SIMT kernel is faster there (measured: C4-d10 iterations
     // 5-7, C4-d5 / C2 late iterations).  Singletons (occ ~ 1) and fully collapsed clusters
     // (occ >= 50: whole-cell summaries) stay on the tensor cores.
-    if (occ > 1.1 && occ < 50.0) {
+    // The slot lists are int32-indexed and cost 4 B per (tile, entry): beyond 2^30 slots
+    // (e.g. C5 iteration 1: 2.5e10 entries, 3e12 pairs) the SIMT kernel runs instead; so it
+    // does when the tiles average less than one entry tile (a CTA per nearly empty tile:
+    // C5 iteration 3, 13 entries per tile, 14 ms vs 2 ms).
+    if ((occ > 1.1 && occ < 50.0) || ent_u + (unsigned long long)owned * kTcEnt > (1ull << 30) ||
+        ent_u < (unsigned long long)owned * kTcEnt) {
       ws.tc_used = 0;
       return run_update_simt<D>(ws, lo, hi, nbr);
     }

@@ -203,6 +203,33 @@ def test_c3_cluster_terminal_property(c3):
     assert oracle.terminal_violations(r["coords"], c.eps, lab, idx) == 0
 
 
+# ------------------------------------------------------------ full-size (C5, one GPU)
+@pytest.fixture(scope="module")
+def c5():
+    c = datagen.CONFIGS["C5"]
+    return c, c.generate(0)
+
+
+def test_c5_first_step_sampled(c5):
+    """BASELINE config C5 at full size on one GPU (n=10M, d=3: ~564k neighbours per point,
+    2.5e10 plan entries, so the update falls back from the tensor-core slot lists to the SIMT
+    kernel): sampled point updates and neighbour counts equal the oracle's definition."""
+    c, X = c5
+    g = E.step(X, c.eps, nbr=True)
+    idx = np.random.default_rng(0).choice(len(X), 48, replace=False)
+    Xs, ns = oracle.step_sample(X, c.eps, idx)
+    assert np.array_equal(g["nbr"][idx], ns)
+    assert np.abs(g["points"][idx].astype(np.float64) - Xs).max() <= 2e-6
+
+
+def test_c5_cluster_terminal_property(c5):
+    c, X = c5
+    r = E.cluster(X, c.eps, coords=True)
+    assert r["converged"]
+    idx = np.random.default_rng(1).choice(len(X), 32, replace=False)
+    assert oracle.terminal_violations(r["coords"], c.eps, r["labels"], idx) == 0
+
+
 def test_pack_unpack_roundtrip_multi_rank_layout():
     """The all-gather plumbing kernels: packing 3 rank ranges of D^{t+1} and unpacking the
     concatenated (ranks*d, cnt) buffer reproduces the next state exactly (bitwise, ragged tail)."""
