@@ -39,7 +39,8 @@ def _step_compare(X, eps, atol=2e-6):
 
 @pytest.mark.parametrize("seed", [0, 1, 2])
 @pytest.mark.parametrize("n,d,k,eps", [(1000, 2, 5, 0.05), (3000, 3, 4, 0.08), (2500, 5, 6, 0.1),
-                                       (4000, 10, 5, 0.2), (777, 7, 3, 0.15), (1500, 1, 3, 0.02)])
+                                       (4000, 10, 5, 0.2), (777, 7, 3, 0.15), (1500, 1, 3, 0.02),
+                                       (2000, 12, 4, 0.25), (1800, 11, 3, 0.25)])
 def test_step_parity(seed, n, d, k, eps):
     _step_compare(datagen.blobs(n, d, k, seed=seed), eps)
 
