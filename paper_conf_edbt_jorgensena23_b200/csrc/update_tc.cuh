@@ -392,9 +392,6 @@ struct TcArgs {
   unsigned long long* prof;  // optional cycle accounting (EGGSYNC_TC_PROF)
 };
 
-__device__ __forceinline__ void named_bar(int id, int cnt) {
-  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(cnt) : "memory");
-}
 
 // shared-memory header of the TC kernel
 struct TcMisc {
