@@ -85,8 +85,8 @@ struct TcCfg {
   static constexpr int kRareBytes = 2 * (NV + 1) * kTcTile * 8;
   static constexpr int kMiscBytes = 3072;
   static constexpr int kBudget = 227 * 1024 - 1024;
-  static constexpr int kStages =
-      (kBudget - kRawBytes - kRareBytes - kMiscBytes) / kStageBytes >= 3 ? 3 : 2;
+  static constexpr int kStages0 = (kBudget - kRawBytes - kRareBytes - kMiscBytes) / kStageBytes;
+  static constexpr int kStages = kStages0 >= 4 ? 4 : (kStages0 >= 3 ? 3 : 2);
   static constexpr int kRingBytes = kStages * kStageBytes;
   static constexpr int kNS = kNS0 < kStages ? kNS0 : kStages;  // the MMA loop needs stages >= S buffers
   static constexpr int kColO = K1 + kNS * kTcEnt;   // O buffers: kColO + N2*g
@@ -395,7 +395,7 @@ struct TcArgs {
 
 // shared-memory header of the TC kernel
 struct TcMisc {
-  uint64_t stage_full[3], stage_empty[3], s_full[3], p_full[3], o_full[2];  // s_full / p_full: per S buffer
+  uint64_t stage_full[4], stage_empty[4], s_full[3], p_full[3], o_full[2];  // s_full / p_full: per S buffer
   uint32_t tbase;
   float o[kTcMaxD], s0[kTcMaxD], c0[kTcMaxD];
   float lo[4][kTcMaxD], hi[4][kTcMaxD];
