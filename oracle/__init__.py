@@ -53,6 +53,8 @@ def lib():
         L.oracle_step_sample.restype = ctypes.c_int
         L.oracle_terminal_sample.argtypes = [vp, i64, i32, f32, vp, vp, i64]
         L.oracle_terminal_sample.restype = ctypes.c_int64
+        L.oracle_order_parameter.argtypes = [vp, i64, i32, f32, vp, vp]
+        L.oracle_order_parameter.restype = ctypes.c_int
         _lib = L
     return _lib
 
@@ -85,6 +87,21 @@ def step(X, eps: float, compute_f2: bool = False):
     if rc != OK:
         raise RuntimeError(f"oracle_step rc={rc}")
     return Xn, nbr, tuple(int(f) for f in flags)
+
+
+def order_parameter(X, eps: float):
+    """Cluster order parameter r_c of the state X (Eq.2, Alg 1 l.6 L54).
+
+    Returns (r_c, per-point inner means) in fp64.
+    """
+    X = np.ascontiguousarray(X, dtype=np.float64)
+    n, d = X.shape
+    out = np.zeros(1, np.float64)
+    rcp = np.empty(n, np.float64)
+    rc = lib().oracle_order_parameter(_p(X), n, d, ctypes.c_float(eps), _p(out), _p(rcp))
+    if rc != OK:
+        raise RuntimeError(f"oracle_order_parameter rc={rc}")
+    return float(out[0]), rcp
 
 
 def cluster(X32, eps: float, term_mode: int = GRID, max_iters: int = 10000):

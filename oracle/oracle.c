@@ -172,6 +172,45 @@ int oracle_step(const double *X, int64_t n, int32_t d, float eps32, double *Xn,
     return ORACLE_OK;
 }
 
+/* ------------------------------------------------------- order parameter */
+
+/*
+ * Cluster order parameter of the state D^t (Eq.2; Alg 1 l.6 L54, SynC's
+ * lambda-termination input, L77/L95):
+ *   r_c = 1/|D| * sum_{p in D} 1/|N_eps(p^t)| * sum_{q in N_eps(p^t)} exp(-||q^t - p^t||)
+ * with N_eps as in R4 (fp64, dimension order, p in N_eps(p)).
+ *   rcp : n, receives the inner mean for every p (may be NULL)
+ * The outer mean is summed serially in point order.
+ */
+int oracle_order_parameter(const double *X, int64_t n, int32_t d, float eps32, double *rc_out,
+                           double *rcp) {
+    if (!X || !rc_out || n < 1 || d < 1) return ORACLE_EINVAL;
+    double C[7];
+    oracle_constants(eps32, d, C);
+    const double e2 = C[1];
+    double *inner = (double *)malloc((size_t)n * sizeof(double));
+    if (!inner) return ORACLE_ENOMEM;
+#pragma omp parallel for schedule(dynamic, 16)
+    for (int64_t p = 0; p < n; ++p) {
+        double s = 0.0;
+        int64_t cnt = 0;
+        for (int64_t q = 0; q < n; ++q) {
+            double dd = sqdist(X, p, q, d);
+            if (dd <= e2) {        /* q in N_eps(p), L66 */
+                ++cnt;
+                s = s + exp(-sqrt(dd));
+            }
+        }
+        inner[p] = s / (double)cnt;
+    }
+    double tot = 0.0;
+    for (int64_t p = 0; p < n; ++p) tot = tot + inner[p];
+    *rc_out = tot / (double)n;
+    if (rcp) memcpy(rcp, inner, (size_t)n * sizeof(double));
+    free(inner);
+    return ORACLE_OK;
+}
+
 /* ------------------------------------------------------------- labelling */
 
 /* canonical relabel: ids numbered by first occurrence in point order (R14) */

@@ -361,3 +361,56 @@ def test_generator_recipe():
     assert a.min() == 0.0 and a.max() == 1.0
     assert np.array_equal(a, b)
     assert not np.array_equal(a, datagen.blobs(5000, 4, 5, noise=0.1, seed=2))
+
+
+# ------------------------------------------------ Eq.2 cluster order parameter
+def test_order_parameter_closed_forms():
+    """Eq.2 L74: isolated points give 1 (N={p}, e^0); a mutually-close pair gives (1+e^-a)/2;
+    a chain 0, a, 2a (2a > eps) gives ((1+e^-a)/2 * 2 + (1+2e^-a)/3) / 3 (pins p in N(p),
+    the 1/|N| inner mean, the 1/|D| outer mean, e^{-||.||} not e^{-||.||^2})."""
+    X = np.array([[0.1, 0.1], [0.9, 0.9], [0.1, 0.9]], np.float32)
+    r, rcp = oracle.order_parameter(X, 0.05)
+    assert r == 1.0 and rcp.tolist() == [1.0, 1.0, 1.0]
+    P = np.array([[0.5, 0.5], [0.52, 0.53]], np.float32)
+    Pd = P.astype(np.float64)
+    a = math.sqrt(((Pd[1] - Pd[0]) ** 2).sum())
+    r, rcp = oracle.order_parameter(P, 0.05)
+    assert r == pytest.approx((1 + math.exp(-a)) / 2, abs=1e-15)
+    # pair + isolated point
+    r, _ = oracle.order_parameter(np.vstack([P, [[0.9, 0.1]]]), 0.05)
+    assert r == pytest.approx(((1 + math.exp(-a)) + 1) / 3, abs=1e-15)
+    # chain: middle point sees both ends, the ends see only the middle
+    C = np.array([[0.0], [0.03], [0.06]], np.float64)
+    r, rcp = oracle.order_parameter(C, 0.05)
+    e0, e1 = (1 + math.exp(-0.03)) / 2, (1 + 2 * math.exp(-0.03)) / 3
+    assert rcp == pytest.approx([e0, e1, e0], abs=1e-15)
+    assert r == pytest.approx((2 * e0 + e1) / 3, abs=1e-15)
+
+
+def test_order_parameter_coincident_and_invariants():
+    """Coincident neighbourhoods give r_c = 1 (L77 'r_c approach 1 when synchronized');
+    0 < r_c <= 1; permutation invariance."""
+    X = np.repeat(np.array([[0.2, 0.4, 0.6], [0.7, 0.1, 0.3]], np.float32), 5, axis=0)
+    assert oracle.order_parameter(X, 0.05)[0] == 1.0
+    Y = datagen.blobs(300, 3, 4, seed=5)
+    r, rcp = oracle.order_parameter(Y, 0.08)
+    assert 0.0 < r <= 1.0 and (rcp > 0).all() and (rcp <= 1).all()
+    perm = np.random.default_rng(1).permutation(len(Y))
+    r2, rcp2 = oracle.order_parameter(Y[perm], 0.08)
+    assert r2 == pytest.approx(r, abs=1e-13)
+    assert np.allclose(rcp2, rcp[perm], atol=1e-14, rtol=0)
+
+
+def test_order_parameter_two_point_convergence():
+    """App.D L392 + Eq.2: for a pair the gap g obeys g' = g - sin g, so r_c = (1+e^-|g|)/2
+    rises towards 1 but never reaches it (L77, L95: 'r_c = 1 is never reached')."""
+    X = np.array([[0.30, 0.60], [0.33, 0.58]], np.float64)
+    g = X[1] - X[0]
+    prev = 0.0
+    for _ in range(3):  # gaps 3.6e-2, 7.8e-6, 8e-17: e^-|g| rounds to 1 after that
+        r, _ = oracle.order_parameter(X, 0.05)
+        assert r == pytest.approx((1 + math.exp(-math.sqrt((g ** 2).sum()))) / 2, abs=1e-14)
+        assert prev < r and (r < 1.0 or math.sqrt((g ** 2).sum()) < 1e-15)
+        prev = r
+        X, _, _ = oracle.step(X, 0.05)
+        g = g - np.sin(g)
