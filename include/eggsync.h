@@ -234,6 +234,53 @@ int64_t eggsync_ctx_owned_count(eggsync_ctx *ctx, int32_t ranks);
 int eggsync_ctx_pack_owned(eggsync_ctx *ctx, int32_t rank, int32_t ranks, float *buf);
 int eggsync_ctx_unpack_owned(eggsync_ctx *ctx, const float *gathered, int32_t ranks);
 
+/* ------------------------------------------------------------------------
+ * Direct SynC (GPU-SynC-style) cross-check and the cluster order parameter
+ * (SURVEY.md §8(f) F4).  No grid, no Eq.5 identity: every point is tested
+ * against every point (O(n^2 d) per update), as the GPU-SynC baseline the
+ * paper compares against does (L284: "distribute updates of all points among
+ * threads").  A second, independent GPU path for Eq.1 and a speed floor for
+ * the grid path; not used by eggsync_cluster.
+ * ---------------------------------------------------------------------- */
+
+/*
+ * eggsync_sync_step -- one synchronous Eq.1 update (L68, Alg 1 l.3-5 L50-53)
+ * computed directly, plus the cluster order parameter of the input state
+ * (Eq.2, Alg 1 l.6 L54):
+ *   r_c = 1/n * sum_p 1/|N_eps(p^t)| * sum_{q in N_eps(p^t)} exp(-||q^t - p^t||).
+ *   points    : in D^t, out D^{t+1}; n*d float32 row-major; device memory when
+ *               on_device = 1 (runs on the legacy default stream), else host.
+ *               Coordinates are used as given (no [0,1] check: Eq.1 needs no grid).
+ *   n, d, eps : 1 <= n <= 2^31-1, 1 <= d <= EGGSYNC_MAX_D, eps finite > 0.
+ *   rc_out    : host double, r_c of D^t (may be NULL).
+ *   nbr_out   : n int32, |N_eps(p^t)| (device when on_device, else host; may be NULL).
+ * N_eps membership (||p-q|| <= eps, p in N_eps(p), L66) is decided exactly: fp32
+ * distances outside a (4d+16)u relative band around eps^2 decide directly, the
+ * rest are re-decided in fp64 as sum_i (q_i - p_i)^2 in dimension order.  Sums of
+ * sin(q_i - p_i) (fp32 sinf) and exp(-||.||) (fp32) are accumulated per 128-point
+ * tile in fp32 and in fp64 across tiles; the update and the mean are fp64 -> the
+ * output float32.  Allocates O(n*d) device scratch per call.  Synchronises.
+ * Returns EGGSYNC_OK, EGGSYNC_EINVAL, EGGSYNC_ENOMEM or EGGSYNC_ECUDA.
+ */
+int eggsync_sync_step(float *points, int64_t n, int32_t d, float eps, int32_t on_device, double *rc_out,
+                      int32_t *nbr_out);
+
+/*
+ * eggsync_sync_lambda -- SynC with lambda-termination (Algorithm 1, L46-56),
+ * GPU-SynC style: repeat { r_c = Eq.2 on D^t; D^{t+1} = Eq.1(D^t); t += 1 }
+ * while r_c < lambda and t < max_iters (the update of the iteration whose r_c
+ * reaches lambda is applied, as Alg 1 l.5-6 order it).  The paper's point
+ * (Fig 1 L89, L95) is that this stops before the exact criterion holds; the
+ * state returned in points can be handed to eggsync_step to see it.
+ *   points, n, d, eps, on_device : as eggsync_sync_step.
+ *   lambda    : threshold (Böhm et al. use 0.999, L77); max_iters >= 1.
+ *   iters_out : updates applied (host, may be NULL); rc_out : last r_c (host, may be NULL).
+ * Returns EGGSYNC_OK when r_c >= lambda was reached, EGGSYNC_NOT_CONVERGED at
+ * max_iters, or a negative error code.
+ */
+int eggsync_sync_lambda(float *points, int64_t n, int32_t d, float eps, double lambda, int32_t max_iters,
+                        int32_t on_device, int32_t *iters_out, double *rc_out);
+
 #ifdef __cplusplus
 }
 #endif

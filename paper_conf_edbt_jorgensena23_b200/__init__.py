@@ -6,7 +6,7 @@ in include/eggsync.h).  This package holds its thin ctypes binding
 input generator (:mod:`.datagen`).  Importing the package does not load the
 library; the first call does, and fails loudly if it is missing.
 """
-from .eggsync import (EggSyncError, Context, cluster, step, lib, last_error,  # noqa: F401
+from .eggsync import (EggSyncError, Context, cluster, step, sync_step, sync_lambda, lib, last_error,  # noqa: F401
                       OK, NOT_CONVERGED, EINVAL, EDOMAIN, ENOMEM, ECUDA, ENCCL, MAX_D)
 
-__all__ = ["EggSyncError", "Context", "cluster", "step", "lib", "last_error"]
+__all__ = ["EggSyncError", "Context", "cluster", "step", "sync_step", "sync_lambda", "lib", "last_error"]

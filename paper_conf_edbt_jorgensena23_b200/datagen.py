@@ -86,3 +86,14 @@ def uniform(n: int, d: int, seed: int = 0) -> np.ndarray:
     """Uniform [0,1]^d points (edge-case tests: no cluster structure)."""
     rng = np.random.default_rng(seed)
     return np.ascontiguousarray(rng.random((n, d)).astype(np.float32))
+
+
+def bridge(m: int = 200, b: int = 3, seed: int = 0) -> np.ndarray:
+    """Fig 1 (L89) shaped input: two tight 2-D clusters of m points (std 0.002) at x = 0.40
+    and 0.48 (0.08 apart, more than eps = 0.05) and a small bridge of b points at x = 0.44,
+    within eps of both.  Used with eps = 0.05 to show lambda-termination stopping early."""
+    rng = np.random.default_rng(seed)
+    a = np.c_[rng.normal(0.40, 0.002, m), rng.normal(0.5, 0.002, m)]
+    c = np.c_[rng.normal(0.48, 0.002, m), rng.normal(0.5, 0.002, m)]
+    br = np.c_[np.full(b, 0.44) + rng.normal(0, 0.001, b), np.full(b, 0.5)]
+    return np.ascontiguousarray(np.vstack([a, c, br]).astype(np.float32))

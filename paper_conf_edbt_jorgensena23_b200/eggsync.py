@@ -27,7 +27,7 @@ SYMBOLS = [
     "eggsync_ctx_unpack", "eggsync_ctx_advance", "eggsync_ctx_labels", "eggsync_ctx_coords",
     "eggsync_ctx_run", "eggsync_ctx_stream", "eggsync_ctx_work", "eggsync_ctx_tc_work", "eggsync_ctx_launches",
     "eggsync_release_cache", "eggsync_ctx_update_owned", "eggsync_ctx_owned_count", "eggsync_ctx_pack_owned",
-    "eggsync_ctx_unpack_owned",
+    "eggsync_ctx_unpack_owned", "eggsync_sync_step", "eggsync_sync_lambda",
 ]
 
 
@@ -99,6 +99,8 @@ def lib():
             "eggsync_ctx_owned_count": ([vp, i32], ctypes.c_int64),
             "eggsync_ctx_pack_owned": ([vp, i32, i32, vp], ctypes.c_int),
             "eggsync_ctx_unpack_owned": ([vp, vp, i32], ctypes.c_int),
+            "eggsync_sync_step": ([vp, i64, i32, f32, i32, vp, vp], ctypes.c_int),
+            "eggsync_sync_lambda": ([vp, i64, i32, f32, ctypes.c_double, i32, i32, vp, vp], ctypes.c_int),
         }
         for name, (args, res) in sig.items():
             fn = getattr(L, name)
@@ -201,6 +203,51 @@ def step(points, eps: float, *, nbr: bool = False):
     if nbr:
         out["nbr"] = cnt
     return out
+
+
+def _sync_points(points):
+    """(array to pass, n, d, on_device): device tensors in place, host arrays copied (never aliased)."""
+    if _is_torch_cuda(points):
+        import torch
+        assert points.dtype == torch.float32 and points.is_contiguous() and points.dim() == 2
+        return points, points.shape[0], points.shape[1], 1
+    x = _host_points(points, writable=True)
+    return x, x.shape[0], x.shape[1], 0
+
+
+def sync_step(points, eps: float, *, nbr: bool = False):
+    """Direct (GPU-SynC-style, no grid) Eq.1 update + Eq.2 r_c of the input (eggsync_sync_step).
+
+    Host numpy input: returns a new array; CUDA tensor input: updated in place.
+    Returns dict(points, rc[, nbr]).
+    """
+    x, n, d, dev = _sync_points(points)
+    cnt = None
+    if nbr:
+        if dev:
+            import torch
+            cnt = torch.empty(n, dtype=torch.int32, device=x.device)
+        else:
+            cnt = np.empty(n, np.int32)
+    rc = ctypes.c_double(0.0)
+    _check(lib().eggsync_sync_step(_ptr(x), n, d, ctypes.c_float(eps), dev, ctypes.byref(rc),
+                                   _ptr(cnt) if nbr else None))
+    out = {"points": x, "rc": rc.value}
+    if nbr:
+        out["nbr"] = cnt
+    return out
+
+
+def sync_lambda(points, eps: float, lam: float = 0.999, *, max_iters: int = 10000):
+    """SynC with lambda-termination (Alg 1) on the GPU (eggsync_sync_lambda).
+
+    Returns dict(points, iters, rc, reached) -- reached is False when max_iters stopped it.
+    """
+    x, n, d, dev = _sync_points(points)
+    it, rc = ctypes.c_int32(0), ctypes.c_double(0.0)
+    r = _check(lib().eggsync_sync_lambda(_ptr(x), n, d, ctypes.c_float(eps), ctypes.c_double(lam), max_iters,
+                                         dev, ctypes.byref(it), ctypes.byref(rc)), (OK, NOT_CONVERGED))
+    return {"points": x, "iters": it.value, "rc": rc.value, "reached": r == OK}
 
 
 class Context:

@@ -84,3 +84,29 @@ def test_no_cpu_fallback_without_device(cuda_available):
         E.cluster(np.full((8, 2), 0.5, np.float32), 0.05)
     assert ei.value.rc == E.ECUDA
     assert "no CUDA device" in str(ei.value)
+
+
+@pytest.mark.parametrize("n,d,eps", [(0, 2, 0.05), (10, 0, 0.05), (10, 33, 0.05), (10, 2, 0.0),
+                                     (10, 2, float("nan")), (2 ** 31, 2, 0.05)])
+def test_sync_entry_points_validate_before_touching_outputs(n, d, eps):
+    """eggsync_sync_step / eggsync_sync_lambda (F4) reject bad sizes with EINVAL, outputs untouched."""
+    pts = np.full((2, 2), 0.5, np.float32)
+    rc = ctypes.c_double(-3.0)
+    it = ctypes.c_int32(-9)
+    L = E.lib()
+    assert L.eggsync_sync_step(pts.ctypes.data_as(ctypes.c_void_p), n, d, ctypes.c_float(eps), 0,
+                               ctypes.byref(rc), None) == E.EINVAL
+    assert L.eggsync_sync_lambda(pts.ctypes.data_as(ctypes.c_void_p), n, d, ctypes.c_float(eps),
+                                 ctypes.c_double(0.999), 10, 0, ctypes.byref(it), ctypes.byref(rc)) == E.EINVAL
+    assert rc.value == -3.0 and it.value == -9 and (pts == 0.5).all()
+    assert L.eggsync_sync_step(None, 10, 2, ctypes.c_float(0.05), 0, None, None) == E.EINVAL
+
+
+def test_sync_lambda_rejects_bad_loop_arguments(cuda_available):
+    if cuda_available:
+        pytest.skip("device present: covered by the GPU tests")
+    pts = np.full((4, 2), 0.5, np.float32)
+    # without a device the call fails loudly (no CPU fallback) before the loop arguments matter
+    with pytest.raises(E.EggSyncError) as ei:
+        E.sync_step(pts, 0.05)
+    assert ei.value.rc == E.ECUDA

@@ -414,3 +414,21 @@ def test_order_parameter_two_point_convergence():
         prev = r
         X, _, _ = oracle.step(X, 0.05)
         g = g - np.sin(g)
+
+
+def test_lambda_termination_stops_early_on_fig1_input():
+    """Fig 1 (L89) / L95 / L298: Alg 1's r_c >= lambda (lambda = 0.999, L77) stops after 2
+    updates on a bridge input whose state still fails Def 4.2 term (i) (the bridge points are
+    eps-close to both clusters), while the exact criterion runs on until one cluster remains."""
+    X = datagen.bridge()
+    cur, t, r = X.copy(), 0, 0.0
+    while r < 0.999:  # Alg 1 l.2-7 (r_c on D^t, update applied in the same iteration)
+        r, _ = oracle.order_parameter(cur, 0.05)
+        Xn, _, f = oracle.step(cur, 0.05)
+        cur, t = Xn.astype(np.float32), t + 1
+    assert t == 2 and 0.999 <= r < 0.9995
+    _, _, f = oracle.step(cur, 0.05)
+    assert f[0] == 0 and f[1] == 0  # not synchronized (Def 4.2 term i fails)
+    res = oracle.cluster(X, 0.05)
+    assert res["rc"] == oracle.OK and res["iters"] > 10
+    assert len(set(res["labels"].tolist())) == 1
