@@ -45,10 +45,17 @@ def lib():
         vp = ctypes.c_void_p
         L.oracle_constants.argtypes = [f32, i32, vp]
         L.oracle_constants.restype = None
+        f64 = ctypes.c_double
+        L.oracle_constants_cw.argtypes = [f32, i32, f64, vp]
+        L.oracle_constants_cw.restype = None
         L.oracle_step.argtypes = [vp, i64, i32, f32, vp, vp, vp, i32]
         L.oracle_step.restype = ctypes.c_int
+        L.oracle_step_cw.argtypes = [vp, i64, i32, f32, f64, vp, vp, vp, i32]
+        L.oracle_step_cw.restype = ctypes.c_int
         L.oracle_cluster.argtypes = [vp, i64, i32, f32, i32, i32, vp, vp, vp, vp]
         L.oracle_cluster.restype = ctypes.c_int
+        L.oracle_cluster_cw.argtypes = [vp, i64, i32, f32, f64, i32, i32, vp, vp, vp, vp]
+        L.oracle_cluster_cw.restype = ctypes.c_int
         L.oracle_step_sample.argtypes = [vp, i64, i32, f32, vp, i64, vp, vp]
         L.oracle_step_sample.restype = ctypes.c_int
         L.oracle_terminal_sample.argtypes = [vp, i64, i32, f32, vp, vp, i64]
@@ -63,15 +70,15 @@ def _p(a: np.ndarray):
     return a.ctypes.data_as(ctypes.c_void_p)
 
 
-def constants(eps: float, d: int) -> dict:
-    """eps, eps^2, c_w (L252), 1/c_w, w (Eq.4), delta (L110), (eps+delta)^2."""
+def constants(eps: float, d: int, cw_factor: float = 1.0) -> dict:
+    """eps, eps^2, c_w (L252, times cw_factor), 1/c_w, w (Eq.4), delta (L110), (eps+delta)^2."""
     out = np.zeros(7, np.float64)
-    lib().oracle_constants(ctypes.c_float(eps), d, _p(out))
+    lib().oracle_constants_cw(ctypes.c_float(eps), d, cw_factor, _p(out))
     keys = ["eps", "eps2", "cw", "inv_cw", "w", "delta", "ed2"]
     return dict(zip(keys, out.tolist()))
 
 
-def step(X, eps: float, compute_f2: bool = False):
+def step(X, eps: float, compute_f2: bool = False, cw_factor: float = 1.0):
     """One Eq.1 update of the state X (n x d; fp32 or fp64, converted to fp64).
 
     Returns (Xn fp64, nbr int32, flags) with flags = (F1_grid, F1_def42, F2);
@@ -82,8 +89,8 @@ def step(X, eps: float, compute_f2: bool = False):
     Xn = np.empty_like(X)
     nbr = np.empty(n, np.int32)
     flags = np.zeros(3, np.int32)
-    rc = lib().oracle_step(_p(X), n, d, ctypes.c_float(eps), _p(Xn), _p(nbr), _p(flags),
-                           int(compute_f2))
+    rc = lib().oracle_step_cw(_p(X), n, d, ctypes.c_float(eps), cw_factor, _p(Xn), _p(nbr), _p(flags),
+                              int(compute_f2))
     if rc != OK:
         raise RuntimeError(f"oracle_step rc={rc}")
     return Xn, nbr, tuple(int(f) for f in flags)
@@ -104,7 +111,7 @@ def order_parameter(X, eps: float):
     return float(out[0]), rcp
 
 
-def cluster(X32, eps: float, term_mode: int = GRID, max_iters: int = 10000):
+def cluster(X32, eps: float, term_mode: int = GRID, max_iters: int = 10000, cw_factor: float = 1.0):
     """Full clustering by the definition.  Returns dict(rc, X, labels, iters, cell_labels)."""
     X32 = np.ascontiguousarray(X32, dtype=np.float32)
     n, d = X32.shape
@@ -112,8 +119,8 @@ def cluster(X32, eps: float, term_mode: int = GRID, max_iters: int = 10000):
     labels = np.empty(n, np.int32)
     cells = np.empty(n, np.int32)
     iters = np.zeros(1, np.int32)
-    rc = lib().oracle_cluster(_p(X32), n, d, ctypes.c_float(eps), term_mode, max_iters,
-                              _p(Xo), _p(labels), _p(iters), _p(cells))
+    rc = lib().oracle_cluster_cw(_p(X32), n, d, ctypes.c_float(eps), cw_factor, term_mode, max_iters,
+                                 _p(Xo), _p(labels), _p(iters), _p(cells))
     if rc < 0 and rc != EPARTITION:
         raise RuntimeError(f"oracle_cluster rc={rc}")
     return {"rc": rc, "X": Xo, "labels": labels, "iters": int(iters[0]), "cell_labels": cells}

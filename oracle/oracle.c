@@ -45,9 +45,10 @@
 
 /* out[0]=eps (as fp64 of the fp32 value), out[1]=eps^2, out[2]=c_w,
  * out[3]=1/c_w, out[4]=w, out[5]=delta, out[6]=(eps+delta)^2            */
-void oracle_constants(float eps32, int32_t d, double *out) {
+void oracle_constants_cw(float eps32, int32_t d, double cw_factor, double *out) {
     double e = (double)eps32;
-    double cw = e / (2.0 * sqrt((double)d));          /* L252: c_w <= sqrt((eps/2)^2/d) */
+    /* L252: c_w <= sqrt((eps/2)^2/d); cw_factor in (0,1] picks a width below the bound (R1) */
+    double cw = cw_factor * (e / (2.0 * sqrt((double)d)));
     double inv_cw = 1.0 / cw;
     double w = ceil(1.0 / cw);                        /* Eq.4: ceil(1/c_w) cells per dim */
     double delta = e - e * sqrt(15.0 / 16.0) + e / 2.0 - sin(e / 2.0); /* L110 */
@@ -59,6 +60,8 @@ void oracle_constants(float eps32, int32_t d, double *out) {
     out[5] = delta;
     out[6] = (e + delta) * (e + delta);
 }
+
+void oracle_constants(float eps32, int32_t d, double *out) { oracle_constants_cw(eps32, d, 1.0, out); }
 
 /* squared Euclidean distance, dimension order, no contraction (R4) */
 static double sqdist(const double *X, int64_t p, int64_t q, int32_t d) {
@@ -98,11 +101,11 @@ static int same_cell(const double *X, int64_t p, int64_t q, int32_t d, double in
  *                         dist(MBR(N_{eps/2}(q)), p) <= eps   (Def 4.2 term ii, L108-110)
  *                         evaluated iff compute_f2 or flags[0] or flags[1]; else -1
  */
-int oracle_step(const double *X, int64_t n, int32_t d, float eps32, double *Xn,
-                int32_t *nbr, int32_t *flags, int32_t compute_f2) {
-    if (!X || !Xn || !flags || n < 1 || d < 1) return ORACLE_EINVAL;
+int oracle_step_cw(const double *X, int64_t n, int32_t d, float eps32, double cw_factor, double *Xn,
+                   int32_t *nbr, int32_t *flags, int32_t compute_f2) {
+    if (!X || !Xn || !flags || n < 1 || d < 1 || !(cw_factor > 0.0 && cw_factor <= 1.0)) return ORACLE_EINVAL;
     double C[7];
-    oracle_constants(eps32, d, C);
+    oracle_constants_cw(eps32, d, cw_factor, C);
     const double e2 = C[1], inv_cw = C[3], ed2 = C[6];
     const int64_t w = (int64_t)C[4];
     const double e2h = e2 / 4.0; /* (eps/2)^2 */
@@ -170,6 +173,11 @@ int oracle_step(const double *X, int64_t n, int32_t d, float eps32, double *Xn,
     free(lo);
     free(hi);
     return ORACLE_OK;
+}
+
+int oracle_step(const double *X, int64_t n, int32_t d, float eps32, double *Xn,
+                int32_t *nbr, int32_t *flags, int32_t compute_f2) {
+    return oracle_step_cw(X, n, d, eps32, 1.0, Xn, nbr, flags, compute_f2);
 }
 
 /* ------------------------------------------------------- order parameter */
@@ -304,12 +312,13 @@ static void cell_partition(const double *X, int64_t n, int32_t d, double inv_cw,
  * Returns ORACLE_OK, ORACLE_NOT_CONVERGED (max_iters reached), ORACLE_EPARTITION
  * when GRID termination's cell partition differs from the eps-components.
  */
-int oracle_cluster(const float *X32, int64_t n, int32_t d, float eps32, int32_t term_mode,
-                   int32_t max_iters, double *X_out, int32_t *labels, int32_t *iters,
-                   int32_t *cell_labels) {
+int oracle_cluster_cw(const float *X32, int64_t n, int32_t d, float eps32, double cw_factor,
+                      int32_t term_mode, int32_t max_iters, double *X_out, int32_t *labels,
+                      int32_t *iters, int32_t *cell_labels) {
     if (!X32 || !labels || !iters || n < 1 || d < 1 || max_iters < 1) return ORACLE_EINVAL;
+    if (!(cw_factor > 0.0 && cw_factor <= 1.0)) return ORACLE_EINVAL;
     double C[7];
-    oracle_constants(eps32, d, C);
+    oracle_constants_cw(eps32, d, cw_factor, C);
     const int64_t w = (int64_t)C[4];
     double *X = (double *)malloc((size_t)(n * d) * sizeof(double));
     double *Xn = (double *)malloc((size_t)(n * d) * sizeof(double));
@@ -319,7 +328,7 @@ int oracle_cluster(const float *X32, int64_t n, int32_t d, float eps32, int32_t 
     int32_t t = 0, synced = 0, status = ORACLE_OK;
     for (;;) {
         int32_t f[3];
-        int rc = oracle_step(X, n, d, eps32, Xn, NULL, f, 0);
+        int rc = oracle_step_cw(X, n, d, eps32, cw_factor, Xn, NULL, f, 0);
         if (rc != ORACLE_OK) { status = rc; break; }
         int32_t f1 = term_mode == 0 ? f[0] : f[1];
         synced = f1 && f[2] == 1;
@@ -342,6 +351,12 @@ int oracle_cluster(const float *X32, int64_t n, int32_t d, float eps32, int32_t 
     free(Xn);
     free(cl);
     return status;
+}
+
+int oracle_cluster(const float *X32, int64_t n, int32_t d, float eps32, int32_t term_mode,
+                   int32_t max_iters, double *X_out, int32_t *labels, int32_t *iters,
+                   int32_t *cell_labels) {
+    return oracle_cluster_cw(X32, n, d, eps32, 1.0, term_mode, max_iters, X_out, labels, iters, cell_labels);
 }
 
 /* ------------------------------------------------------ sampled variants */

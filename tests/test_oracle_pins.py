@@ -432,3 +432,36 @@ def test_lambda_termination_stops_early_on_fig1_input():
     res = oracle.cluster(X, 0.05)
     assert res["rc"] == oracle.OK and res["iters"] > 10
     assert len(set(res["labels"].tolist())) == 1
+
+
+# ------------------------------------------- cell width below the L252 bound
+def test_cw_factor_constants():
+    """L252 only bounds c_w <= eps/(2 sqrt d); cw_factor f picks f*eps/(2 sqrt d), w = ceil(1/c_w) (Eq.4)."""
+    c = oracle.constants(0.05, 2, 0.5)
+    assert c["cw"] == pytest.approx(0.5 * 0.05 / (2 * math.sqrt(2)), rel=1e-7)
+    assert c["w"] == math.ceil(1 / c["cw"]) == 114
+    c1 = oracle.constants(0.05, 2)
+    assert c1["w"] == 57 and c["delta"] == c1["delta"] and c["eps2"] == c1["eps2"]
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_cw_factor_same_clustering(seed):
+    """Theorem 4.7 (L133-135) holds for any c_w <= eps/(2 sqrt d): the eps-components of the final
+    state equal the verified state's cell partition (rc OK, no EPARTITION) and the partition is
+    the same as at f = 1.  Halved cells nest in the f = 1 cells, so the grid criterion (L252) is
+    stricter and never stops earlier."""
+    X = datagen.blobs(600, 2, 5, seed=seed)
+    r1 = oracle.cluster(X, 0.05)
+    for f in (0.5, 0.3):
+        rf = oracle.cluster(X, 0.05, cw_factor=f)
+        assert rf["rc"] == oracle.OK
+        assert np.array_equal(rf["labels"], r1["labels"])
+        if f == 0.5:
+            assert rf["iters"] >= r1["iters"]
+
+
+def test_cw_factor_out_of_range():
+    X = np.full((3, 2), 0.5, np.float32)
+    for f in (0.0, 1.5, float("nan")):
+        with pytest.raises(RuntimeError):
+            oracle.cluster(X, 0.05, cw_factor=f)
