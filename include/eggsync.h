@@ -82,6 +82,11 @@ typedef struct eggsync_opts {
   float *coords_out;       /* optional n*d row-major final coordinates (original point order) */
   int32_t *nbr_count_out;  /* optional, step only: |N_eps(p)| on D^t, original order */
   eggsync_stats *stats;    /* optional */
+  double cw_factor;        /* grid cell width c_w = cw_factor * eps / (2 sqrt d); (0, 1], default 1.
+                              L252 only requires c_w <= sqrt((eps/2)^2 / d): any smaller width keeps
+                              the grid first term equivalent to Def 4.2 term (i) and Theorem 4.7's
+                              labels; smaller cells make the criterion stricter (never earlier).
+                              Outside (0, 1] -> EGGSYNC_EINVAL. */
 } eggsync_opts;
 
 /* Fill *o with the defaults above (struct_size set). */

@@ -33,16 +33,20 @@ void set_error(const char* fmt, ...) {
   g_err = buf;
 }
 
-bool make_consts(int64_t n, int d, float eps, Consts* c, std::string* why) {
+bool make_consts(int64_t n, int d, float eps, Consts* c, std::string* why, double cw_factor) {
   if (!(eps > 0.f) || !std::isfinite(eps)) {
     *why = "eps must be finite and > 0";
+    return false;
+  }
+  if (!(cw_factor > 0.0 && cw_factor <= 1.0)) {
+    *why = "cw_factor must be in (0, 1] (c_w <= eps/(2 sqrt d), L252)";
     return false;
   }
   c->n = n;
   c->d = d;
   c->e = (double)eps;
   c->e2 = c->e * c->e;
-  c->cw = c->e / (2.0 * std::sqrt((double)d));  // L252: cell diagonal = eps/2
+  c->cw = cw_factor * (c->e / (2.0 * std::sqrt((double)d)));  // L252: cell diagonal <= eps/2
   c->inv_cw = 1.0 / c->cw;
   const double wd = std::ceil(1.0 / c->cw);     // Eq.4
   if (wd > 2147483647.0) {
@@ -212,9 +216,9 @@ static void cache_clear() {
   if (prev >= 0) cudaSetDevice(prev);
 }
 
-int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st) {
+int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st, double cw_factor) {
   std::string why;
-  if (!make_consts(n_, d_, eps, &k, &why)) {
+  if (!make_consts(n_, d_, eps, &k, &why, cw_factor)) {
     set_error("%s", why.c_str());
     return EGGSYNC_EINVAL;
   }
@@ -584,6 +588,7 @@ void eggsync_default_opts(eggsync_opts* o) {
   o->max_iters = 10000;
   o->device = -1;
   o->term_mode = EGGSYNC_TERM_GRID;
+  o->cw_factor = 1.0;
 }
 
 static int get_opts(const eggsync_opts* in, eggsync_opts* o) {
@@ -596,6 +601,10 @@ static int get_opts(const eggsync_opts* in, eggsync_opts* o) {
   *o = *in;
   if (o->max_iters < 1) {
     set_error("max_iters must be >= 1");
+    return EGGSYNC_EINVAL;
+  }
+  if (!(o->cw_factor > 0.0 && o->cw_factor <= 1.0)) {
+    set_error("cw_factor=%g must be in (0, 1] (c_w <= eps/(2 sqrt d), L252)", o->cw_factor);
     return EGGSYNC_EINVAL;
   }
   if (o->term_mode != EGGSYNC_TERM_GRID) {
@@ -621,7 +630,7 @@ int eggsync_cluster_ex(const float* points, int64_t n, int32_t d, float eps, con
   eggsync_stats* stats = o.stats ? &local : nullptr;
   auto t0 = std::chrono::steady_clock::now();
   Workspace ws;
-  EGG_TRY(ws.alloc(n, d, eps, o.device, (cudaStream_t)o.stream));
+  EGG_TRY(ws.alloc(n, d, eps, o.device, (cudaStream_t)o.stream, o.cw_factor));
   EGG_CUDA(cudaStreamSynchronize(ws.stream));
   auto t1 = std::chrono::steady_clock::now();
   if (stats) stats->t_alloc = std::chrono::duration<double>(t1 - t0).count();
@@ -670,7 +679,7 @@ int eggsync_step_ex(float* points, int64_t n, int32_t d, float eps, const eggsyn
   DeviceGuard g;
   EGG_TRY(g.set(o.device));
   Workspace ws;
-  EGG_TRY(ws.alloc(n, d, eps, o.device, (cudaStream_t)o.stream));
+  EGG_TRY(ws.alloc(n, d, eps, o.device, (cudaStream_t)o.stream, o.cw_factor));
   EGG_TRY(stage_ingest(ws, points, o.device_pointers != 0));
   int32_t synced = 0, f1 = 0, f2 = -1;
   EGG_TRY(iterate(ws, &synced, &f1, &f2, o.nbr_count_out ? ws.nbr : nullptr, nullptr));

@@ -77,7 +77,7 @@ struct Consts {
   float ef, e2f, edf, ed2f, rel;  // fp32 copies; rel = (4d+16) u relative safety margin
 };
 
-bool make_consts(int64_t n, int d, float eps, Consts* c, std::string* why);
+bool make_consts(int64_t n, int d, float eps, Consts* c, std::string* why, double cw_factor = 1.0);
 
 // thread-local error message
 void set_error(const char* fmt, ...);
@@ -241,7 +241,7 @@ struct Workspace {
   cudaEvent_t tc_ev[2] = {nullptr, nullptr};
   int tc_flush();                         // fold a pending launch's event time into tc_acc
 
-  int alloc(int64_t n, int d, float eps, int device, cudaStream_t stream);
+  int alloc(int64_t n, int d, float eps, int device, cudaStream_t stream, double cw_factor = 1.0);
   void release();
   ~Workspace() { release(); }
 };

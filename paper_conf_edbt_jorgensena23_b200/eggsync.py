@@ -53,7 +53,7 @@ class Opts(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_int32), ("max_iters", ctypes.c_int32), ("device", ctypes.c_int32),
                 ("device_pointers", ctypes.c_int32), ("stream", ctypes.c_void_p), ("term_mode", ctypes.c_int32),
                 ("coords_out", ctypes.c_void_p), ("nbr_count_out", ctypes.c_void_p),
-                ("stats", ctypes.POINTER(Stats))]
+                ("stats", ctypes.POINTER(Stats)), ("cw_factor", ctypes.c_double)]
 
 
 _lib = None
@@ -149,7 +149,7 @@ def _host_points(points, writable=False):
 
 
 def cluster(points, eps: float, *, max_iters: int = 10000, coords: bool = False, stats: bool = False,
-            stream=None):
+            stream=None, cw_factor: float = 1.0):
     """EGG-SynC clustering (Alg 4).  points: (n,d) float32 numpy (host) or CUDA torch tensor.
 
     Returns dict(labels, iters, converged[, coords][, stats]).  Device inputs give device outputs.
@@ -157,6 +157,7 @@ def cluster(points, eps: float, *, max_iters: int = 10000, coords: bool = False,
     dev = _is_torch_cuda(points)
     o = default_opts()
     o.max_iters = max_iters
+    o.cw_factor = cw_factor
     if dev:
         import torch
         assert points.dtype == torch.float32 and points.is_contiguous() and points.dim() == 2
@@ -188,11 +189,12 @@ def cluster(points, eps: float, *, max_iters: int = 10000, coords: bool = False,
     return out
 
 
-def step(points, eps: float, *, nbr: bool = False):
+def step(points, eps: float, *, nbr: bool = False, cw_factor: float = 1.0):
     """One Eq.1 update (eggsync_step_ex) of host points.  Returns dict(points, first, second, synced[, nbr])."""
     x = _host_points(points, writable=True)
     n, d = x.shape
     o = default_opts()
+    o.cw_factor = cw_factor
     cnt = np.empty(n, np.int32) if nbr else None
     if nbr:
         o.nbr_count_out = _ptr(cnt)

@@ -39,6 +39,7 @@ def test_default_opts():
     o = E.default_opts()
     assert o.struct_size == ctypes.sizeof(E.Opts)
     assert o.max_iters == 10000 and o.device == -1 and o.device_pointers == 0
+    assert o.cw_factor == 1.0
 
 
 @pytest.mark.parametrize("n,d,eps", [(0, 2, 0.05), (10, 0, 0.05), (10, 33, 0.05), (10, 2, 0.0),
@@ -110,3 +111,17 @@ def test_sync_lambda_rejects_bad_loop_arguments(cuda_available):
     with pytest.raises(E.EggSyncError) as ei:
         E.sync_step(pts, 0.05)
     assert ei.value.rc == E.ECUDA
+
+
+@pytest.mark.parametrize("f", [0.0, -0.5, 1.0000001, float("nan"), float("inf")])
+def test_cw_factor_out_of_range_is_einval(f):
+    """opts.cw_factor must lie in (0, 1] (c_w <= eps/(2 sqrt d), L252); checked before any output."""
+    o = E.default_opts()
+    o.cw_factor = f
+    pts = np.full((4, 2), 0.5, np.float32)
+    lab = np.full(4, -7, np.int32)
+    it = ctypes.c_int32(-9)
+    rc = E.lib().eggsync_cluster_ex(pts.ctypes.data_as(ctypes.c_void_p), 4, 2, ctypes.c_float(0.05),
+                                    ctypes.byref(o), lab.ctypes.data_as(ctypes.c_void_p), ctypes.byref(it))
+    assert rc == E.EINVAL and "cw_factor" in E.last_error()
+    assert (lab == -7).all() and it.value == -9
