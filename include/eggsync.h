@@ -57,6 +57,12 @@ extern "C" {
 
 /* termination modes (ambiguity register R1/F3 in DESIGN.md) */
 #define EGGSYNC_TERM_GRID 0 /* first term via |cell(p)| == |N_eps(p)| (Alg 3 l.14-15 L248, L252) */
+#define EGGSYNC_TERM_DEF42 1 /* Def 4.2 literally (L106-110): term (i) "no pair with eps/2 < ||p-q|| <= eps",
+                                term (ii) with MBR(N_{eps/2}(q)); labels = connected components of
+                                the eps-graph of the returned state (Theorem 4.7).  eggsync_cluster_ex
+                                only; runs on the direct (all-pairs, O(n^2 d) per iteration) kernels of
+                                eggsync_sync_step, not the grid; ignores cw_factor and stats other
+                                than iters. */
 
 /*
  * Per-stage timings of the last call, mirroring the columns of Table 1
@@ -78,7 +84,7 @@ typedef struct eggsync_opts {
   int32_t device;          /* CUDA ordinal; -1 = current device */
   int32_t device_pointers; /* 1: points / labels / coords_out / nbr_count_out are device pointers */
   void *stream;            /* cudaStream_t to run on; NULL = library-owned stream */
-  int32_t term_mode;       /* EGGSYNC_TERM_GRID (only mode implemented) */
+  int32_t term_mode;       /* EGGSYNC_TERM_GRID (default) or EGGSYNC_TERM_DEF42 (cluster_ex only) */
   float *coords_out;       /* optional n*d row-major final coordinates (original point order) */
   int32_t *nbr_count_out;  /* optional, step only: |N_eps(p)| on D^t, original order */
   eggsync_stats *stats;    /* optional */

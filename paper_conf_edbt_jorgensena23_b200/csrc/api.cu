@@ -607,8 +607,8 @@ static int get_opts(const eggsync_opts* in, eggsync_opts* o) {
     set_error("cw_factor=%g must be in (0, 1] (c_w <= eps/(2 sqrt d), L252)", o->cw_factor);
     return EGGSYNC_EINVAL;
   }
-  if (o->term_mode != EGGSYNC_TERM_GRID) {
-    set_error("term_mode %d not implemented (only EGGSYNC_TERM_GRID)", o->term_mode);
+  if (o->term_mode != EGGSYNC_TERM_GRID && o->term_mode != EGGSYNC_TERM_DEF42) {
+    set_error("term_mode %d unknown (EGGSYNC_TERM_GRID or EGGSYNC_TERM_DEF42)", o->term_mode);
     return EGGSYNC_EINVAL;
   }
   return EGGSYNC_OK;
@@ -626,6 +626,7 @@ int eggsync_cluster_ex(const float* points, int64_t n, int32_t d, float eps, con
   EGG_TRY(check_device());
   DeviceGuard g;
   EGG_TRY(g.set(o.device));
+  if (o.term_mode == EGGSYNC_TERM_DEF42) return def42_cluster(points, n, d, eps, o, labels_out, iters_out);
   eggsync_stats local{};
   eggsync_stats* stats = o.stats ? &local : nullptr;
   auto t0 = std::chrono::steady_clock::now();
@@ -674,6 +675,10 @@ int eggsync_step_ex(float* points, int64_t n, int32_t d, float eps, const eggsyn
                     int32_t* first_term_out, int32_t* second_term_out) {
   eggsync_opts o;
   EGG_TRY(get_opts(opts, &o));
+  if (o.term_mode != EGGSYNC_TERM_GRID) {
+    set_error("eggsync_step_ex evaluates the grid criterion only (term_mode must be EGGSYNC_TERM_GRID)");
+    return EGGSYNC_EINVAL;
+  }
   EGG_TRY(validate(points, n, d, eps));
   EGG_TRY(check_device());
   DeviceGuard g;

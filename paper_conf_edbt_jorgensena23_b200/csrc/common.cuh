@@ -79,6 +79,10 @@ struct Consts {
 
 bool make_consts(int64_t n, int d, float eps, Consts* c, std::string* why, double cw_factor = 1.0);
 
+// term_mode = EGGSYNC_TERM_DEF42 clustering on the direct kernels (sync_brute.cu).
+int def42_cluster(const float* points, int64_t n, int d, float eps, const eggsync_opts& o, int32_t* labels_out,
+                  int32_t* iters_out);
+
 // thread-local error message
 void set_error(const char* fmt, ...);
 

@@ -26,7 +26,22 @@ struct SyncArgs {
   int64_t n;
   float e2_lo, e2_hi;  // fp32 band around eps^2: below lo -> in, above hi -> out
   double e2;           // exact test (fp64 of the fp32 eps, squared)
+  int32_t* f1_def;     // Def 4.2 term (i) flag (cleared on a pair eps/2 < ||p-q|| <= eps) or nullptr
+  float e2h_lo, e2h_hi;
+  double e2h;          // (eps/2)^2 = e2 / 4 (as the oracle)
 };
+
+// Exact fp64 squared distance: the oracle's predicate (R4), dimension order, no FMA.
+template <int D>
+__device__ __forceinline__ double exact_d2(const float* q, const float* x) {
+  double dd = 0.0;
+#pragma unroll
+  for (int i = 0; i < D; ++i) {
+    const double t = (double)q[i] - (double)x[i];
+    dd = __dadd_rn(dd, __dmul_rn(t, t));
+  }
+  return dd;
+}
 
 template <int D>
 __global__ void __launch_bounds__(kSyncT) k_sync_brute(SyncArgs a) {
@@ -61,17 +76,11 @@ __global__ void __launch_bounds__(kSyncT) k_sync_brute(SyncArgs a) {
       }
       if (d2 > a.e2_hi) continue;
       bool in = d2 <= a.e2_lo;
-      if (!in) {  // inside the band: the oracle's exact fp64 decision (dimension order, no FMA)
-        double dd = 0.0;
-#pragma unroll
-        for (int i = 0; i < D; ++i) {
-          const double t = (double)q[i] - (double)x[i];
-          dd = __dadd_rn(dd, __dmul_rn(t, t));
-        }
-        in = dd <= a.e2;
-      }
+      if (!in) in = exact_d2<D>(q, x) <= a.e2;  // inside the band: the oracle's exact decision
       if (in) {  // q in N_eps(p): Eq.1 term sin(q_i - p_i), Eq.2 term exp(-||q - p||)
         ++cnt;
+        if (a.f1_def && act && d2 > a.e2h_lo && (d2 > a.e2h_hi || exact_d2<D>(q, x) > a.e2h))
+          *a.f1_def = 0;  // eps/2 < ||p - q|| <= eps: Def 4.2 term (i) fails (L108)
 #pragma unroll
         for (int i = 0; i < D; ++i) s[i] += sinf(q[i] - x[i]);
         r += expf(-sqrtf(d2));
@@ -104,9 +113,9 @@ __global__ void __launch_bounds__(1024) k_mean(const double* __restrict__ v, int
 }
 
 template <int D>
-int launch_sync(const SyncArgs& a) {
+int launch_sync(const SyncArgs& a, cudaStream_t st) {
   const int64_t blocks = (a.n + kSyncT - 1) / kSyncT;
-  k_sync_brute<D><<<(unsigned)blocks, kSyncT>>>(a);
+  k_sync_brute<D><<<(unsigned)blocks, kSyncT, 0, st>>>(a);
   EGG_CUDA(cudaGetLastError());
   return EGGSYNC_OK;
 }
@@ -162,22 +171,331 @@ struct SyncBufs {
 };
 
 // One Alg 1 iteration on device buffers: xn = Eq.1(x), *rc_dev = Eq.2(x).
-int sync_iter(const float* x, float* xn, int32_t* nbr, double* rcp, double* rc_dev, int64_t n, int d, float eps) {
+int sync_iter(const float* x, float* xn, int32_t* nbr, double* rcp, int64_t n, int d, float eps,
+              int32_t* f1_def = nullptr, cudaStream_t st = 0) {
   const double e = (double)eps;
-  const float e2f = (float)(e * e);
+  const double e2 = e * e, e2h = e2 / 4.0;
+  const float e2f = (float)e2, e2hf = (float)e2h;
   const float rel = (float)(4 * d + 16) * kU;
-  SyncArgs a{x, xn, nbr, rcp, n, e2f * (1.f - rel), e2f * (1.f + rel), e * e};
-  EGG_DISPATCH(d, launch_sync, a);
+  SyncArgs a{x, xn, nbr, rcp, n, e2f * (1.f - rel), e2f * (1.f + rel), e2,
+             f1_def, e2hf * (1.f - rel), e2hf * (1.f + rel), e2h};
+  EGG_DISPATCH(d, launch_sync, a, st);
 }
 
 int sync_run(const float* x, float* xn, int32_t* nbr, double* rcp, double* rc_dev, int64_t n, int d, float eps) {
-  EGG_TRY(sync_iter(x, xn, nbr, rcp, rc_dev, n, d, eps));
+  EGG_TRY(sync_iter(x, xn, nbr, rcp, n, d, eps));
   k_mean<<<1, 1024>>>(rcp, n, rc_dev);
   EGG_CUDA(cudaGetLastError());
   return EGGSYNC_OK;
 }
 
+
+// ============================================================================
+// term_mode = EGGSYNC_TERM_DEF42: Def 4.2 literally (L106-110) on the
+// direct path -- term (i) "no pair with eps/2 < ||p-q|| <= eps" (flag of k_sync_brute),
+// term (ii) with MBR(N_{eps/2}(q)) per point, labels = connected components of the eps-graph
+// (Theorem 4.7: at the criterion they are the clusters).  O(n^2 d) per iteration.
+// ============================================================================
+
+// MBR(N_{eps/2}(q)) of every q: lo/hi [n][D] (min/max of fp32 coordinates: exact).
+template <int D>
+__global__ void __launch_bounds__(kSyncT) k_half_mbr(const float* __restrict__ X, int64_t n, float lo_f, float hi_f,
+                                                     double e2h, float* __restrict__ lo, float* __restrict__ hi) {
+  __shared__ float tile[kSyncT * D];
+  const int64_t p = (int64_t)blockIdx.x * kSyncT + threadIdx.x;
+  const bool act = p < n;
+  float x[D], l[D], h[D];
+#pragma unroll
+  for (int i = 0; i < D; ++i) l[i] = h[i] = x[i] = act ? X[p * D + i] : 0.f;
+  for (int64_t t0 = 0; t0 < n; t0 += kSyncT) {
+    const int64_t rem = n - t0;
+    const int m = rem < kSyncT ? (int)rem : kSyncT;
+    __syncthreads();
+    for (int k = threadIdx.x; k < m * D; k += kSyncT) tile[k] = X[t0 * D + k];
+    __syncthreads();
+    for (int j = 0; j < m; ++j) {
+      const float* q = tile + j * D;
+      float d2 = 0.f;
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        const float t = q[i] - x[i];
+        d2 = fmaf(t, t, d2);
+      }
+      if (d2 > hi_f) continue;
+      if (d2 > lo_f && exact_d2<D>(q, x) > e2h) continue;
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        l[i] = fminf(l[i], q[i]);
+        h[i] = fmaxf(h[i], q[i]);
+      }
+    }
+  }
+  if (!act) return;
+#pragma unroll
+  for (int i = 0; i < D; ++i) {
+    lo[p * D + i] = l[i];
+    hi[p * D + i] = h[i];
+  }
+}
+
+// Def 4.2 term (ii) (L108-110): clear *f2 if some p, q have eps < ||p-q|| <= eps+delta and
+// dist(MBR(N_{eps/2}(q)), p) <= eps (per-dimension clamp distance, R10), all in fp64 as the oracle.
+template <int D>
+__global__ void __launch_bounds__(kSyncT) k_second_def(const float* __restrict__ X, int64_t n,
+                                                       const float* __restrict__ lo, const float* __restrict__ hi,
+                                                       float in_lo, float out_hi, double e2, double ed2,
+                                                       int32_t* __restrict__ f2) {
+  __shared__ float tile[kSyncT * D];
+  const int64_t p = (int64_t)blockIdx.x * kSyncT + threadIdx.x;
+  const bool act = p < n;
+  float x[D];
+#pragma unroll
+  for (int i = 0; i < D; ++i) x[i] = act ? X[p * D + i] : 0.f;
+  bool viol = false;
+  for (int64_t t0 = 0; t0 < n; t0 += kSyncT) {
+    const int64_t rem = n - t0;
+    const int m = rem < kSyncT ? (int)rem : kSyncT;
+    __syncthreads();
+    for (int k = threadIdx.x; k < m * D; k += kSyncT) tile[k] = X[t0 * D + k];
+    __syncthreads();
+    if (!act || viol) continue;
+    for (int j = 0; j < m; ++j) {
+      const float* q = tile + j * D;
+      float d2 = 0.f;
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        const float t = q[i] - x[i];
+        d2 = fmaf(t, t, d2);
+      }
+      if (d2 < in_lo || d2 > out_hi) continue;  // surely inside eps or outside eps + delta
+      const double dd = exact_d2<D>(q, x);
+      if (!(dd > e2 && dd <= ed2)) continue;
+      const int64_t qi = t0 + j;
+      double mm = 0.0;
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        const double v = (double)x[i], L = (double)lo[qi * D + i], H = (double)hi[qi * D + i];
+        double t = 0.0;
+        if (v < L) t = __dsub_rn(L, v);
+        else if (v > H) t = __dsub_rn(v, H);
+        mm = __dadd_rn(mm, __dmul_rn(t, t));
+      }
+      if (mm <= e2) {
+        viol = true;
+        break;
+      }
+    }
+  }
+  if (viol) *f2 = 0;
+}
+
+// One min-label propagation round over the eps-graph: out[p] = min(in[p], in[q] : ||p-q|| <= eps).
+template <int D>
+__global__ void __launch_bounds__(kSyncT) k_cc_round(const float* __restrict__ X, int64_t n, float lo_f, float hi_f,
+                                                     double e2, const int32_t* __restrict__ in,
+                                                     int32_t* __restrict__ out, int32_t* __restrict__ changed) {
+  __shared__ float tile[kSyncT * D];
+  __shared__ int32_t tl[kSyncT];
+  const int64_t p = (int64_t)blockIdx.x * kSyncT + threadIdx.x;
+  const bool act = p < n;
+  float x[D];
+#pragma unroll
+  for (int i = 0; i < D; ++i) x[i] = act ? X[p * D + i] : 0.f;
+  int32_t m = act ? in[p] : 0;
+  for (int64_t t0 = 0; t0 < n; t0 += kSyncT) {
+    const int64_t rem = n - t0;
+    const int mm = rem < kSyncT ? (int)rem : kSyncT;
+    __syncthreads();
+    for (int k = threadIdx.x; k < mm * D; k += kSyncT) tile[k] = X[t0 * D + k];
+    if ((int)threadIdx.x < mm) tl[threadIdx.x] = in[t0 + threadIdx.x];
+    __syncthreads();
+    for (int j = 0; j < mm; ++j) {
+      if (tl[j] >= m) continue;
+      const float* q = tile + j * D;
+      float d2 = 0.f;
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        const float t = q[i] - x[i];
+        d2 = fmaf(t, t, d2);
+      }
+      if (d2 > hi_f) continue;
+      if (d2 > lo_f && exact_d2<D>(q, x) > e2) continue;
+      m = tl[j];
+    }
+  }
+  if (!act) return;
+  out[p] = m;
+  if (m != in[p]) *changed = 1;
+}
+
+__global__ void k_jump(const int32_t* __restrict__ in, int64_t n, int32_t* __restrict__ out) {
+  const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (p < n) out[p] = in[in[p]];
+}
+
+// Canonical numbering (R14): component label = its smallest index m (lab[m] == m); ids are
+// the ranks of those roots in index order.  One CTA: chunked counts, block scan, scatter.
+__global__ void __launch_bounds__(1024) k_canon(const int32_t* __restrict__ lab, int64_t n, int32_t* __restrict__ ids,
+                                                int32_t* __restrict__ labels) {
+  __shared__ int32_t sc[1024];
+  const int64_t chunk = (n + 1023) / 1024;
+  const int64_t b = threadIdx.x * chunk, e = b + chunk < n ? b + chunk : n;
+  int32_t c = 0;
+  for (int64_t p = b; p < e; ++p) c += lab[p] == p;
+  sc[threadIdx.x] = c;
+  __syncthreads();
+  for (int off = 1; off < 1024; off <<= 1) {
+    const int32_t v = (int)threadIdx.x >= off ? sc[threadIdx.x - off] : 0;
+    __syncthreads();
+    sc[threadIdx.x] += v;
+    __syncthreads();
+  }
+  int32_t id = sc[threadIdx.x] - c;
+  for (int64_t p = b; p < e; ++p)
+    if (lab[p] == p) ids[p] = id++;
+  __syncthreads();
+  for (int64_t p = threadIdx.x; p < n; p += 1024) labels[p] = ids[lab[p]];
+}
+
+__global__ void k_domain(const float* __restrict__ X, int64_t m, int32_t* __restrict__ bad) {
+  const int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (k < m && !(X[k] >= 0.f && X[k] <= 1.f)) *bad = 1;  // NaN fails both comparisons
+}
+__global__ void k_iota(int32_t* __restrict__ v, int64_t n) {
+  const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (p < n) v[p] = (int32_t)p;
+}
+
+template <int D>
+int launch_def42_second(const float* x, int64_t n, float eps, float* lo, float* hi, int32_t* f2, cudaStream_t st) {
+  const double e = (double)eps, e2 = e * e, e2h = e2 / 4.0;
+  const double delta = e - e * std::sqrt(15.0 / 16.0) + e / 2.0 - std::sin(e / 2.0);  // L110 (R11)
+  const double ed2 = (e + delta) * (e + delta);
+  const float rel = (float)(4 * D + 16) * kU;
+  const unsigned blocks = (unsigned)((n + kSyncT - 1) / kSyncT);
+  k_half_mbr<D><<<blocks, kSyncT, 0, st>>>(x, n, (float)e2h * (1.f - rel), (float)e2h * (1.f + rel), e2h, lo, hi);
+  k_second_def<D><<<blocks, kSyncT, 0, st>>>(x, n, lo, hi, (float)e2 * (1.f - rel), (float)ed2 * (1.f + rel), e2, ed2,
+                                             f2);
+  EGG_CUDA(cudaGetLastError());
+  return EGGSYNC_OK;
+}
+
+template <int D>
+int launch_cc_round(const float* x, int64_t n, float eps, const int32_t* in, int32_t* out, int32_t* changed,
+                    cudaStream_t st) {
+  const double e = (double)eps, e2 = e * e;
+  const float rel = (float)(4 * D + 16) * kU;
+  const unsigned blocks = (unsigned)((n + kSyncT - 1) / kSyncT);
+  k_cc_round<D><<<blocks, kSyncT, 0, st>>>(x, n, (float)e2 * (1.f - rel), (float)e2 * (1.f + rel), e2, in, out,
+                                           changed);
+  EGG_CUDA(cudaGetLastError());
+  return EGGSYNC_OK;
+}
+
+int def42_second(const float* x, int64_t n, int d, float eps, float* lo, float* hi, int32_t* f2, cudaStream_t st) {
+  EGG_DISPATCH(d, launch_def42_second, x, n, eps, lo, hi, f2, st);
+}
+int cc_round(const float* x, int64_t n, int d, float eps, const int32_t* in, int32_t* out, int32_t* changed,
+             cudaStream_t st) {
+  EGG_DISPATCH(d, launch_cc_round, x, n, eps, in, out, changed, st);
+}
+
+struct Def42Bufs {
+  float* x[2] = {nullptr, nullptr};
+  float *lo = nullptr, *hi = nullptr;
+  int32_t *lab[2] = {nullptr, nullptr}, *ids = nullptr, *out = nullptr, *flags = nullptr;
+  double* rcp = nullptr;
+  ~Def42Bufs() {
+    for (void* p : {(void*)x[0], (void*)x[1], (void*)lo, (void*)hi, (void*)lab[0], (void*)lab[1], (void*)ids,
+                    (void*)out, (void*)flags, (void*)rcp})
+      cudaFree(p);
+  }
+};
+
+int set_flag(int32_t* f, int32_t v, cudaStream_t st) {
+  EGG_CUDA(cudaMemsetAsync(f, 0, sizeof(int32_t), st));
+  if (v) EGG_CUDA(cudaMemsetAsync(f, 1, 1, st));  // little-endian int32 1
+  return EGGSYNC_OK;
+}
+int get_flag(const int32_t* f, int32_t* v, cudaStream_t st) {
+  EGG_CUDA(cudaMemcpyAsync(v, f, sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+  EGG_CUDA(cudaStreamSynchronize(st));
+  return EGGSYNC_OK;
+}
+
 }  // namespace
+
+// Algorithm 4 (R6/R7) with Def 4.2's literal first term; called by eggsync_cluster_ex for
+// term_mode == EGGSYNC_TERM_DEF42 after argument validation.  Labels: eps-components of the
+// returned state, canonical (as oracle_cluster's DEF42 mode).
+int def42_cluster(const float* points, int64_t n, int d, float eps, const eggsync_opts& o, int32_t* labels_out,
+                  int32_t* iters_out) {
+  cudaStream_t st = (cudaStream_t)o.stream;
+  const bool dev = o.device_pointers != 0;
+  const size_t bytes = sizeof(float) * n * d;
+  Def42Bufs b;
+  EGG_CUDA(cudaMalloc(&b.x[0], bytes));
+  EGG_CUDA(cudaMalloc(&b.x[1], bytes));
+  EGG_CUDA(cudaMalloc(&b.lo, bytes));
+  EGG_CUDA(cudaMalloc(&b.hi, bytes));
+  for (int k = 0; k < 2; ++k) EGG_CUDA(cudaMalloc(&b.lab[k], sizeof(int32_t) * n));
+  EGG_CUDA(cudaMalloc(&b.ids, sizeof(int32_t) * n));
+  EGG_CUDA(cudaMalloc(&b.out, sizeof(int32_t) * n));
+  EGG_CUDA(cudaMalloc(&b.flags, sizeof(int32_t) * 4));
+  EGG_CUDA(cudaMalloc(&b.rcp, sizeof(double) * n));
+  EGG_CUDA(cudaMemcpyAsync(b.x[0], points, bytes, dev ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, st));
+  // domain (L70, L290): every coordinate finite and in [0,1]
+  EGG_TRY(set_flag(b.flags + 3, 0, st));
+  k_domain<<<(unsigned)((n * d + 255) / 256), 256, 0, st>>>(b.x[0], n * d, b.flags + 3);
+  int32_t bad = 0;
+  EGG_TRY(get_flag(b.flags + 3, &bad, st));
+  if (bad) {
+    set_error("a coordinate is NaN/Inf or outside [0,1]");
+    return EGGSYNC_EDOMAIN;
+  }
+  int32_t t = 0, cur = 0, synced = 0;
+  for (;;) {
+    EGG_TRY(set_flag(b.flags, 1, st));
+    EGG_TRY(sync_iter(b.x[cur], b.x[cur ^ 1], nullptr, b.rcp, n, d, eps, b.flags, st));
+    int32_t f1 = 0, f2 = 0;
+    EGG_TRY(get_flag(b.flags, &f1, st));
+    if (f1) {
+      EGG_TRY(set_flag(b.flags + 1, 1, st));
+      EGG_TRY(def42_second(b.x[cur], n, d, eps, b.lo, b.hi, b.flags + 1, st));
+      EGG_TRY(get_flag(b.flags + 1, &f2, st));
+    }
+    synced = f1 && f2;
+    cur ^= 1;
+    ++t;
+    if (synced || t >= o.max_iters) break;
+  }
+  // eps-components of the returned state: min-label propagation + pointer jumping
+  const unsigned nb = (unsigned)((n + 255) / 256);
+  k_iota<<<nb, 256, 0, st>>>(b.lab[0], n);
+  for (;;) {
+    EGG_TRY(set_flag(b.flags + 2, 0, st));
+    EGG_TRY(cc_round(b.x[cur], n, d, eps, b.lab[0], b.lab[1], b.flags + 2, st));
+    k_jump<<<nb, 256, 0, st>>>(b.lab[1], n, b.lab[0]);
+    EGG_CUDA(cudaGetLastError());
+    int32_t ch = 0;
+    EGG_TRY(get_flag(b.flags + 2, &ch, st));
+    if (!ch) break;
+  }
+  k_canon<<<1, 1024, 0, st>>>(b.lab[0], n, b.ids, b.out);
+  EGG_CUDA(cudaGetLastError());
+  EGG_CUDA(cudaMemcpyAsync(labels_out, b.out, sizeof(int32_t) * n, dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
+                           st));
+  if (o.coords_out)
+    EGG_CUDA(cudaMemcpyAsync(o.coords_out, b.x[cur], bytes, dev ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, st));
+  EGG_CUDA(cudaStreamSynchronize(st));
+  if (o.stats) {
+    memset(o.stats, 0, sizeof(eggsync_stats));
+    o.stats->iters = t;
+  }
+  *iters_out = t;
+  return synced ? EGGSYNC_OK : EGGSYNC_NOT_CONVERGED;
+}
+
 }  // namespace egg
 
 using namespace egg;

@@ -148,8 +148,11 @@ def _host_points(points, writable=False):
     return a.copy() if writable else a  # step() writes D^{t+1}: never alias the caller's array
 
 
+TERM_GRID, TERM_DEF42 = 0, 1
+
+
 def cluster(points, eps: float, *, max_iters: int = 10000, coords: bool = False, stats: bool = False,
-            stream=None, cw_factor: float = 1.0):
+            stream=None, cw_factor: float = 1.0, term_mode: int = TERM_GRID):
     """EGG-SynC clustering (Alg 4).  points: (n,d) float32 numpy (host) or CUDA torch tensor.
 
     Returns dict(labels, iters, converged[, coords][, stats]).  Device inputs give device outputs.
@@ -158,6 +161,7 @@ def cluster(points, eps: float, *, max_iters: int = 10000, coords: bool = False,
     o = default_opts()
     o.max_iters = max_iters
     o.cw_factor = cw_factor
+    o.term_mode = term_mode
     if dev:
         import torch
         assert points.dtype == torch.float32 and points.is_contiguous() and points.dim() == 2

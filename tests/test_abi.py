@@ -125,3 +125,20 @@ def test_cw_factor_out_of_range_is_einval(f):
                                     ctypes.byref(o), lab.ctypes.data_as(ctypes.c_void_p), ctypes.byref(it))
     assert rc == E.EINVAL and "cw_factor" in E.last_error()
     assert (lab == -7).all() and it.value == -9
+
+
+def test_term_mode_validation():
+    """term_mode: GRID (0) or DEF42 (1, cluster_ex only); anything else EINVAL before any output."""
+    pts = np.full((4, 2), 0.5, np.float32)
+    lab = np.full(4, -7, np.int32)
+    it = ctypes.c_int32(-9)
+    o = E.default_opts()
+    o.term_mode = 2
+    rc = E.lib().eggsync_cluster_ex(pts.ctypes.data_as(ctypes.c_void_p), 4, 2, ctypes.c_float(0.05),
+                                    ctypes.byref(o), lab.ctypes.data_as(ctypes.c_void_p), ctypes.byref(it))
+    assert rc == E.EINVAL and (lab == -7).all() and it.value == -9
+    o.term_mode = E.TERM_DEF42
+    f1, f2 = ctypes.c_int32(-3), ctypes.c_int32(-3)
+    rc = E.lib().eggsync_step_ex(pts.ctypes.data_as(ctypes.c_void_p), 4, 2, ctypes.c_float(0.05), ctypes.byref(o),
+                                 ctypes.byref(f1), ctypes.byref(f2))
+    assert rc == E.EINVAL and f1.value == -3 and (pts == 0.5).all()
