@@ -212,10 +212,16 @@ def step(points, eps: float, *, nbr: bool = False, cw_factor: float = 1.0):
 
 
 def _sync_points(points):
-    """(array to pass, n, d, on_device): device tensors in place, host arrays copied (never aliased)."""
+    """(array to pass, n, d, on_device): device tensors in place, host arrays copied (never aliased).
+
+    The direct-path entry points run on the legacy default stream of the current device:
+    a device tensor's device becomes current and its producer stream is drained first.
+    """
     if _is_torch_cuda(points):
         import torch
         assert points.dtype == torch.float32 and points.is_contiguous() and points.dim() == 2
+        torch.cuda.set_device(points.device)
+        torch.cuda.current_stream(points.device).synchronize()
         return points, points.shape[0], points.shape[1], 1
     x = _host_points(points, writable=True)
     return x, x.shape[0], x.shape[1], 0
