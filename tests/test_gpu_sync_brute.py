@@ -100,3 +100,29 @@ def test_lambda_max_iters():
     X = datagen.bridge()
     g = E.sync_lambda(X, 0.05, 1.5, max_iters=3)  # r_c <= 1 < lambda: runs to max_iters
     assert not g["reached"] and g["iters"] == 3
+
+
+def test_sync_step_c3_full_size_sampled():
+    """C3 at full size (n = 1,000,000, d = 10): 96 sampled point updates and r_c terms of the
+    direct path against the oracle's per-point definition (oracle_step_sample)."""
+    c = datagen.make_config("C3")
+    X = datagen.blobs(c.n, c.d, c.k, noise=c.noise, seed=0)
+    g = E.sync_step(X, c.eps, nbr=True)
+    idx = np.random.default_rng(11).choice(c.n, 96, replace=False)
+    Xo, nbr_o = oracle.step_sample(X, c.eps, idx)
+    assert np.array_equal(g["nbr"][idx], nbr_o)
+    assert np.abs(g["points"][idx].astype(np.float64) - Xo).max() <= 2e-6
+    assert 0.0 < g["rc"] < 1.0
+
+
+@pytest.mark.parametrize("seed", [0, 1])
+def test_lambda_loop_c1_matches_oracle(seed):
+    X = datagen.blobs(1000, 2, 5, seed=seed)
+    g = E.sync_lambda(X, 0.05, 0.999)
+    cur, t, r = X.copy(), 0, 0.0
+    while r < 0.999:
+        r, _ = oracle.order_parameter(cur, 0.05)
+        Xn, _, _ = oracle.step(cur, 0.05)
+        cur, t = Xn.astype(np.float32), t + 1
+    assert g["reached"] and g["iters"] == t and abs(g["rc"] - r) <= 1e-6
+    assert np.abs(g["points"].astype(np.float64) - cur).max() <= 1e-5
