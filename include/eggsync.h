@@ -61,7 +61,8 @@ extern "C" {
                                 term (ii) with MBR(N_{eps/2}(q)); labels = connected components of
                                 the eps-graph of the returned state (Theorem 4.7).  eggsync_cluster_ex
                                 only; runs on the direct (all-pairs, O(n^2 d) per iteration) kernels of
-                                eggsync_sync_step, not the grid; ignores cw_factor and stats other
+                                eggsync_sync_step, not the grid, on opts.stream (NULL: the
+                                legacy default stream); ignores cw_factor and stats other
                                 than iters. */
 
 /*
