@@ -45,12 +45,15 @@ __device__ __forceinline__ double exact_d2(const float* q, const float* x) {
 
 template <int D>
 __global__ void __launch_bounds__(kSyncT) k_sync_brute(SyncArgs a) {
-  __shared__ float tile[kSyncT * D];
+  constexpr int DP = ceil4(D);  // tile rows padded to whole float4s (pads are 0 in q and p)
+  __shared__ float4 tile4[kSyncT * DP / 4];
+  __shared__ uint8_t hq[kSyncT * kSyncT];  // [slot k][thread]: neighbour queue of the current tile
+  float* tile = reinterpret_cast<float*>(tile4);
   const int64_t p = (int64_t)blockIdx.x * kSyncT + threadIdx.x;
   const bool act = p < a.n;
-  float x[D];
+  float x[DP];
 #pragma unroll
-  for (int i = 0; i < D; ++i) x[i] = act ? a.x[p * D + i] : 0.f;
+  for (int i = 0; i < DP; ++i) x[i] = (act && i < D) ? a.x[p * D + i] : 0.f;
   double S[D];
 #pragma unroll
   for (int i = 0; i < D; ++i) S[i] = 0.0;
@@ -60,31 +63,55 @@ __global__ void __launch_bounds__(kSyncT) k_sync_brute(SyncArgs a) {
     const int64_t rem = a.n - t0;
     const int m = rem < kSyncT ? (int)rem : kSyncT;
     __syncthreads();
-    for (int k = threadIdx.x; k < m * D; k += kSyncT) tile[k] = a.x[t0 * D + k];
+    for (int k = threadIdx.x; k < m * D; k += kSyncT) tile[(k / D) * DP + (k % D)] = a.x[t0 * D + k];
+    if (DP != D)
+      for (int k = threadIdx.x; k < m * (DP - D); k += kSyncT) tile[(k / (DP - D)) * DP + D + k % (DP - D)] = 0.f;
     __syncthreads();
+    // pass 1: the pair test (float4 shared loads, broadcast); each thread queues the tile
+    // slots of its neighbours in ascending order
+    int nh = 0;
+    for (int j = 0; j < m; ++j) {
+      const float4* q4 = tile4 + j * (DP / 4);
+      float d2 = 0.f;
+#pragma unroll
+      for (int c = 0; c < DP / 4; ++c) {
+        const float4 v = q4[c];
+        float t = v.x - x[4 * c];
+        d2 = fmaf(t, t, d2);
+        t = v.y - x[4 * c + 1];
+        d2 = fmaf(t, t, d2);
+        t = v.z - x[4 * c + 2];
+        d2 = fmaf(t, t, d2);
+        t = v.w - x[4 * c + 3];
+        d2 = fmaf(t, t, d2);
+      }
+      if (d2 > a.e2_hi) continue;
+      const float* q = tile + j * DP;
+      bool in = d2 <= a.e2_lo;
+      if (!in) in = exact_d2<D>(q, x) <= a.e2;  // inside the band: the oracle's exact decision
+      if (in) {
+        hq[nh++ * kSyncT + threadIdx.x] = (uint8_t)j;
+        if (a.f1_def && act && d2 > a.e2h_lo && (d2 > a.e2h_hi || exact_d2<D>(q, x) > a.e2h))
+          *a.f1_def = 0;  // eps/2 < ||p - q|| <= eps: Def 4.2 term (i) fails (L108)
+      }
+    }
+    // pass 2: q in N_eps(p): Eq.1 terms sin(q_i - p_i), Eq.2 term exp(-||q - p||).  The warp
+    // runs max(nh) iterations over its lanes instead of one sinf branch per slot any lane hits.
+    cnt += nh;
     float s[D];
 #pragma unroll
     for (int i = 0; i < D; ++i) s[i] = 0.f;
     float r = 0.f;
-    for (int j = 0; j < m; ++j) {
-      const float* q = tile + j * D;
+    for (int k = 0; k < nh; ++k) {
+      const float* q = tile + (int)hq[k * kSyncT + threadIdx.x] * DP;
       float d2 = 0.f;
 #pragma unroll
       for (int i = 0; i < D; ++i) {
         const float t = q[i] - x[i];
         d2 = fmaf(t, t, d2);
+        s[i] += sinf(t);
       }
-      if (d2 > a.e2_hi) continue;
-      bool in = d2 <= a.e2_lo;
-      if (!in) in = exact_d2<D>(q, x) <= a.e2;  // inside the band: the oracle's exact decision
-      if (in) {  // q in N_eps(p): Eq.1 term sin(q_i - p_i), Eq.2 term exp(-||q - p||)
-        ++cnt;
-        if (a.f1_def && act && d2 > a.e2h_lo && (d2 > a.e2h_hi || exact_d2<D>(q, x) > a.e2h))
-          *a.f1_def = 0;  // eps/2 < ||p - q|| <= eps: Def 4.2 term (i) fails (L108)
-#pragma unroll
-        for (int i = 0; i < D; ++i) s[i] += sinf(q[i] - x[i]);
-        r += expf(-sqrtf(d2));
-      }
+      r += expf(-sqrtf(d2));
     }
 #pragma unroll
     for (int i = 0; i < D; ++i) S[i] += (double)s[i];
