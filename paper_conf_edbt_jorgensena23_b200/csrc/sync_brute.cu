@@ -29,6 +29,8 @@ struct SyncArgs {
   int32_t* f1_def;     // Def 4.2 term (i) flag (cleared on a pair eps/2 < ||p-q|| <= eps) or nullptr
   float e2h_lo, e2h_hi;
   double e2h;          // (eps/2)^2 = e2 / 4 (as the oracle)
+  int64_t qchunk;      // q points per slice (blockIdx.y); slices > 1 write partial sums to part
+  double* part;        // [slice][n][D+2]: sum sin, sum exp, count (nullptr when one slice)
 };
 
 // Exact fp64 squared distance: the oracle's predicate (R4), dimension order, no FMA.
@@ -59,12 +61,14 @@ __global__ void __launch_bounds__(kSyncT) k_sync_brute(SyncArgs a) {
   for (int i = 0; i < D; ++i) S[i] = 0.0;
   double R = 0.0;
   int32_t cnt = 0;
-  for (int64_t t0 = 0; t0 < a.n; t0 += kSyncT) {
-    const int64_t rem = a.n - t0;
+  const int64_t q0 = (int64_t)blockIdx.y * a.qchunk;
+  const int64_t q1 = q0 + a.qchunk < a.n ? q0 + a.qchunk : a.n;
+  for (int64_t t0 = q0; t0 < q1; t0 += kSyncT) {
+    const int64_t rem = q1 - t0;
     const int m = rem < kSyncT ? (int)rem : kSyncT;
     __syncthreads();
     for (int k = threadIdx.x; k < m * D; k += kSyncT) tile[(k / D) * DP + (k % D)] = a.x[t0 * D + k];
-    if (DP != D)
+    if constexpr (DP != D)
       for (int k = threadIdx.x; k < m * (DP - D); k += kSyncT) tile[(k / (DP - D)) * DP + D + k % (DP - D)] = 0.f;
     __syncthreads();
     // pass 1: the pair test (float4 shared loads, broadcast); each thread queues the tile
@@ -118,11 +122,40 @@ __global__ void __launch_bounds__(kSyncT) k_sync_brute(SyncArgs a) {
     R += (double)r;
   }
   if (!act) return;
+  if (a.part) {  // one slice of the q range: partial sums, combined in slice order by k_sync_reduce
+    double* o = a.part + ((int64_t)blockIdx.y * a.n + p) * (D + 2);
+#pragma unroll
+    for (int i = 0; i < D; ++i) o[i] = S[i];
+    o[D] = R;
+    o[D + 1] = (double)cnt;
+    return;
+  }
   const double inv = 1.0 / (double)cnt;  // cnt >= 1: p in N_eps(p)
 #pragma unroll
   for (int i = 0; i < D; ++i) a.xn[p * D + i] = (float)((double)x[i] + inv * S[i]);
   if (a.nbr) a.nbr[p] = cnt;
   a.rcp[p] = R * inv;
+}
+
+// Sum of the slices' partial sums in slice order (deterministic) + Eq.1 / Eq.2 epilogue.
+template <int D>
+__global__ void k_sync_reduce(SyncArgs a, int slices) {
+  const int64_t p = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (p >= a.n) return;
+  double S[D + 2];
+#pragma unroll
+  for (int i = 0; i < D + 2; ++i) S[i] = 0.0;
+  for (int sl = 0; sl < slices; ++sl) {
+    const double* o = a.part + ((int64_t)sl * a.n + p) * (D + 2);
+#pragma unroll
+    for (int i = 0; i < D + 2; ++i) S[i] += o[i];
+  }
+  const int32_t cnt = (int32_t)S[D + 1];
+  const double inv = 1.0 / (double)cnt;
+#pragma unroll
+  for (int i = 0; i < D; ++i) a.xn[p * D + i] = (float)((double)a.x[p * D + i] + inv * S[i]);
+  if (a.nbr) a.nbr[p] = cnt;
+  a.rcp[p] = S[D] * inv;
 }
 
 // Deterministic mean of the per-point inner means (one CTA, fixed order).
@@ -139,11 +172,31 @@ __global__ void __launch_bounds__(1024) k_mean(const double* __restrict__ v, int
   if (threadIdx.x == 0) *out = sh[0] / (double)n;
 }
 
+// Slices of the q range: one thread per p gives only ceil(n/128) CTAs, too few to fill 148 SMs
+// below n ~ 100k; split the q range so about 6 CTAs per SM run (each slice >= 1 tile).
+int64_t sync_slices(int64_t n) {
+  const int64_t nb = (n + kSyncT - 1) / kSyncT;
+  int64_t sl = (148 * 6 + nb - 1) / nb;
+  if (sl > nb) sl = nb;
+  if (sl > 64) sl = 64;
+  return sl < 1 ? 1 : sl;
+}
+
 template <int D>
-int launch_sync(const SyncArgs& a, cudaStream_t st) {
+int launch_sync(SyncArgs a, cudaStream_t st) {
   const int64_t blocks = (a.n + kSyncT - 1) / kSyncT;
-  k_sync_brute<D><<<(unsigned)blocks, kSyncT, 0, st>>>(a);
+  const int64_t sl = sync_slices(a.n);
+  a.qchunk = ((a.n + sl - 1) / sl + kSyncT - 1) / kSyncT * kSyncT;
+  const int64_t used = (a.n + a.qchunk - 1) / a.qchunk;
+  a.part = nullptr;
+  if (used > 1) EGG_CUDA(cudaMallocAsync(&a.part, sizeof(double) * used * a.n * (D + 2), st));
+  k_sync_brute<D><<<dim3((unsigned)blocks, (unsigned)used), kSyncT, 0, st>>>(a);
   EGG_CUDA(cudaGetLastError());
+  if (used > 1) {
+    k_sync_reduce<D><<<(unsigned)((a.n + 255) / 256), 256, 0, st>>>(a, (int)used);
+    EGG_CUDA(cudaGetLastError());
+    EGG_CUDA(cudaFreeAsync(a.part, st));
+  }
   return EGGSYNC_OK;
 }
 
@@ -205,7 +258,7 @@ int sync_iter(const float* x, float* xn, int32_t* nbr, double* rcp, int64_t n, i
   const float e2f = (float)e2, e2hf = (float)e2h;
   const float rel = (float)(4 * d + 16) * kU;
   SyncArgs a{x, xn, nbr, rcp, n, e2f * (1.f - rel), e2f * (1.f + rel), e2,
-             f1_def, e2hf * (1.f - rel), e2hf * (1.f + rel), e2h};
+             f1_def, e2hf * (1.f - rel), e2hf * (1.f + rel), e2h, n, nullptr};
   EGG_DISPATCH(d, launch_sync, a, st);
 }
 
