@@ -280,6 +280,23 @@ def run_ours(args):
                       "(workspace alloc/free, H2D, all iterations, D2H)"}
     if world == 1 and not args.no_cpu:
         cpu = cpu_baseline_obj(X, c, args.cpu_seconds)
+    # context (not the metric): one direct all-pairs Eq.1 update (GPU-SynC style, F4) of the same
+    # D^0 on the same GPU, against the grid path's mean iteration of the timed clusterings
+    direct = None
+    if world == 1 and not args.no_direct:
+        Xd0 = torch.from_numpy(X).cuda()
+        tds = []
+        for k in range(2):
+            u = Xd0.clone()
+            torch.cuda.synchronize()
+            t0 = time.perf_counter()
+            E.sync_step(u, c.eps)  # synchronous (reads r_c back)
+            if k:
+                tds.append((time.perf_counter() - t0) * 1e3)
+        direct = {"ms_per_iteration": tds[0], "grid_ms_per_iteration": ms / iters,
+                  "grid_speedup": tds[0] / (ms / iters),
+                  "how": "wall time of one synchronous eggsync_sync_step on device-resident D^0 (k_sync_brute, "
+                         "O(n^2 d), scratch alloc included, 1 warm-up); grid = ms_per_step / iters"}
     if rank != 0:
         return
     line = {
@@ -295,6 +312,7 @@ def run_ours(args):
                    "launches_per_step": launches / args.steps, "work_counters": work},
         "roofline": roof,
         "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches, "clocks": clk_s,
+        "direct_path_context": direct,
     }
     print(json.dumps(line), flush=True)
     if world > 1:
@@ -344,6 +362,7 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-direct", action="store_true", help="skip the direct-path (GPU-SynC-style) context timing")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
