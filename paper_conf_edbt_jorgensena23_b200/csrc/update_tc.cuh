@@ -129,7 +129,10 @@ struct PlanArgs {
   int32_t* flags;
 };
 
-constexpr int kPlanWarps = 4;
+#ifndef EGG_PLAN_WARPS
+#define EGG_PLAN_WARPS 4
+#endif
+constexpr int kPlanWarps = EGG_PLAN_WARPS;  // point tiles (one warp each) per plan CTA
 
 __device__ __forceinline__ int64_t tc_tile_base(int64_t lo, int64_t tile, int32_t stride, int32_t offset) {
   return lo + (tile * stride + offset) * (int64_t)kTcTile;
