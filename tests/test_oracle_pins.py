@@ -174,7 +174,11 @@ def test_worked_examples(name):
     if "first_step_flags" in g:
         _, _, f = oracle.step(X, g["eps"], compute_f2=True)
         ff = g["first_step_flags"]
-        assert f == (ff["F1_grid"], ff["F1_def42"], ff["F2"])
+        assert f == (ff["F1_grid"], ff["F1_def42"], ff["F2"]), g["cite"]
+    if "def42_iters" in g:
+        r4 = oracle.cluster(X, g["eps"], term_mode=oracle.DEF42)
+        assert r4["rc"] == oracle.OK and r4["iters"] == g["def42_iters"], g["cite"]
+        assert r4["labels"].tolist() == g["labels"], g["cite"]
 
 
 def test_bridge_chain_first_step_closed_form():
