@@ -37,6 +37,19 @@ def _stale(obj, src):
     return any(os.path.getmtime(f) > t for f in [src] + _headers())
 
 
+def _flags_stamp() -> None:
+    """Objects built with other flags (e.g. another EGG_NVCC_EXTRA -D knob) are stale: the
+    flag set is recorded in the build directory and a change removes every object."""
+    stamp = os.path.join(BUILD, "flags.txt")
+    want = " ".join([NVCC, *ARCH, *FLAGS])
+    have = open(stamp).read() if os.path.exists(stamp) else None
+    if have != want:
+        for f in glob.glob(os.path.join(BUILD, "*.o")):
+            os.remove(f)
+        with open(stamp, "w") as fh:
+            fh.write(want)
+
+
 def _compile(src, verbose_ptxas=False):
     obj = os.path.join(BUILD, os.path.basename(src)[:-3] + ".o")
     if not _stale(obj, src):
@@ -56,6 +69,7 @@ def build(force: bool = False, verbose_ptxas: bool = False, jobs: int | None = N
     if force:
         for f in glob.glob(os.path.join(BUILD, "*.o")):
             os.remove(f)
+    _flags_stamp()
     jobs = jobs or max(1, min(len(srcs), os.cpu_count() or 4))
     with cf.ThreadPoolExecutor(jobs) as ex:
         results = list(ex.map(lambda s: _compile(s, verbose_ptxas), srcs))

@@ -255,6 +255,7 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st, do
       {(void**)&c_hi, sizeof(uint32_t) * d * cap},
       {(void**)&c_cnt, sizeof(int32_t) * cap},
       {(void**)&c_rec, sizeof(float) * CREC * cap},
+      {(void**)&c_dig, d <= kTcMaxD ? (size_t)(((kDigMax * (2 * d + 1)) + 15) / 16 * 16) * cap : 0},
       {(void**)&c_key, sizeof(uint64_t) * nw * cap},
       {(void**)&t_meta, sizeof(int4) * cap},
       {(void**)&t_parent, sizeof(int32_t) * cap},
@@ -574,6 +575,11 @@ struct eggsync_ctx {
   Workspace ws;
 };
 
+// every context entry point runs on the context's device and restores the caller's
+#define CTX_DEVICE(ctx)  \
+  DeviceGuard _ctx_dg; \
+  EGG_TRY(_ctx_dg.set((ctx)->ws.cur_device))
+
 extern "C" {
 
 const char* eggsync_last_error(void) { return g_err.c_str(); }
@@ -723,7 +729,8 @@ int eggsync_ctx_create(int64_t n, int32_t d, float eps, int32_t device, void* st
   static const float dummy = 0.f;
   EGG_TRY(validate(&dummy, n, d, eps));
   EGG_TRY(check_device());
-  if (device >= 0) EGG_CUDA(cudaSetDevice(device));
+  DeviceGuard g;  // the caller's current device is restored on return
+  EGG_TRY(g.set(device));
   eggsync_ctx* c = new eggsync_ctx();
   int rc = c->ws.alloc(n, d, eps, device, (cudaStream_t)stream);
   if (rc != EGGSYNC_OK) {
@@ -734,15 +741,22 @@ int eggsync_ctx_create(int64_t n, int32_t d, float eps, int32_t device, void* st
   return EGGSYNC_OK;
 }
 
-void eggsync_ctx_destroy(eggsync_ctx* ctx) { delete ctx; }
+void eggsync_ctx_destroy(eggsync_ctx* ctx) {
+  if (!ctx) return;
+  DeviceGuard g;
+  g.set(ctx->ws.cur_device);
+  delete ctx;
+}
 
 int eggsync_ctx_load(eggsync_ctx* ctx, const float* points, int32_t on_device) {
   if (!ctx || !points) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   return stage_ingest(ctx->ws, points, on_device != 0);
 }
 
 int eggsync_ctx_build(eggsync_ctx* ctx, int32_t* n_cells_out) {
   if (!ctx) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   Workspace& ws = ctx->ws;
   EGG_TRY(stage_build(ws));
   k_set_flags<<<1, 1, 0, ws.stream>>>(ws.flags, 1, 1);
@@ -755,6 +769,7 @@ int eggsync_ctx_build(eggsync_ctx* ctx, int32_t* n_cells_out) {
 
 int eggsync_ctx_update(eggsync_ctx* ctx, int64_t lo, int64_t hi) {
   if (!ctx || lo < 0 || hi > ctx->ws.n || lo > hi) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   if (!ctx->ws.built) {
     set_error("eggsync_ctx_update before eggsync_ctx_build");
     return EGGSYNC_EINVAL;
@@ -764,6 +779,7 @@ int eggsync_ctx_update(eggsync_ctx* ctx, int64_t lo, int64_t hi) {
 
 int eggsync_ctx_second_term(eggsync_ctx* ctx, int64_t lo, int64_t hi) {
   if (!ctx || lo < 0 || hi > ctx->ws.n || lo > hi) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   if (!ctx->ws.built) return EGGSYNC_EINVAL;
   ctx->ws.second_checked = true;
   return stage_second_term(ctx->ws, lo, hi);
@@ -771,6 +787,7 @@ int eggsync_ctx_second_term(eggsync_ctx* ctx, int64_t lo, int64_t hi) {
 
 int eggsync_ctx_flags(eggsync_ctx* ctx, int32_t* first_out, int32_t* second_out) {
   if (!ctx) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   int32_t f1 = 0, f2 = 0;
   EGG_TRY(read_flags(ctx->ws, &f1, &f2, nullptr));
   if (first_out) *first_out = f1;
@@ -783,6 +800,7 @@ float* eggsync_ctx_next_coords(eggsync_ctx* ctx) { return ctx ? ctx->ws.xs[ctx->
 
 int eggsync_ctx_pack(eggsync_ctx* ctx, int64_t lo, int64_t cnt, float* buf) {
   if (!ctx || !buf || lo < 0 || cnt < 0) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   Workspace& ws = ctx->ws;
   const int64_t tot = cnt * ws.d;
   if (tot == 0) return EGGSYNC_OK;
@@ -794,6 +812,7 @@ int eggsync_ctx_pack(eggsync_ctx* ctx, int64_t lo, int64_t cnt, float* buf) {
 
 int eggsync_ctx_unpack(eggsync_ctx* ctx, const float* gathered, int32_t ranks, int64_t cnt) {
   if (!ctx || !gathered || ranks < 1 || cnt < 0) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   Workspace& ws = ctx->ws;
   const int64_t tot = (int64_t)ranks * ws.d * cnt;
   if (tot == 0) return EGGSYNC_OK;
@@ -806,6 +825,7 @@ int eggsync_ctx_unpack(eggsync_ctx* ctx, const float* gathered, int32_t ranks, i
 
 int eggsync_ctx_advance(eggsync_ctx* ctx) {
   if (!ctx) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   advance(ctx->ws);
   ctx->ws.have_final = false;
   return EGGSYNC_OK;
@@ -813,6 +833,7 @@ int eggsync_ctx_advance(eggsync_ctx* ctx) {
 
 int eggsync_ctx_labels(eggsync_ctx* ctx, int32_t* labels, int32_t on_device) {
   if (!ctx || !labels) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   Workspace& ws = ctx->ws;
   const int32_t* src = ws.lab_final;
   if (!ws.have_final) {
@@ -828,6 +849,7 @@ int eggsync_ctx_labels(eggsync_ctx* ctx, int32_t* labels, int32_t on_device) {
 
 int eggsync_ctx_coords(eggsync_ctx* ctx, float* coords, int32_t on_device) {
   if (!ctx || !coords) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   Workspace& ws = ctx->ws;
   if (on_device) {
     EGG_TRY(stage_coords(ws, ws.xcur, coords));
@@ -841,6 +863,7 @@ int eggsync_ctx_coords(eggsync_ctx* ctx, float* coords, int32_t on_device) {
 
 int eggsync_ctx_run(eggsync_ctx* ctx, int32_t max_iters, int32_t* iters_out) {
   if (!ctx || !iters_out || max_iters < 1) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   return run_loop(ctx->ws, max_iters, iters_out, nullptr);
 }
 
@@ -848,6 +871,7 @@ void* eggsync_ctx_stream(eggsync_ctx* ctx) { return ctx ? (void*)ctx->ws.stream 
 
 int eggsync_ctx_work(eggsync_ctx* ctx, int32_t enable, int64_t* totals_out) {
   if (!ctx) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   Workspace& ws = ctx->ws;
   if (totals_out) {
     EGG_CUDA(cudaMemcpyAsync(totals_out, ws.work, 8 * sizeof(int64_t), cudaMemcpyDeviceToHost, ws.stream));
@@ -878,6 +902,7 @@ int Workspace::tc_flush() {
 
 int eggsync_ctx_tc_work(eggsync_ctx* ctx, int32_t enable, int64_t* out) {
   if (!ctx) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   Workspace& ws = ctx->ws;
   EGG_TRY(ws.tc_flush());
   if (out)
@@ -897,6 +922,7 @@ int eggsync_ctx_tc_work(eggsync_ctx* ctx, int32_t enable, int64_t* out) {
 
 int eggsync_ctx_update_owned(eggsync_ctx* ctx, int32_t rank, int32_t ranks) {
   if (!ctx || ranks < 1 || rank < 0 || rank >= ranks) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   if (!ctx->ws.built) {
     set_error("eggsync_ctx_update_owned before eggsync_ctx_build");
     return EGGSYNC_EINVAL;
@@ -916,6 +942,7 @@ int64_t eggsync_ctx_owned_count(eggsync_ctx* ctx, int32_t ranks) {
 
 int eggsync_ctx_pack_owned(eggsync_ctx* ctx, int32_t rank, int32_t ranks, float* buf) {
   if (!ctx || !buf || ranks < 1 || rank < 0 || rank >= ranks) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   Workspace& ws = ctx->ws;
   const int64_t cnt = owned_count(ws, ranks), tot = cnt * ws.d;
   k_pack_owned<<<(unsigned)((tot + 255) / 256), 256, 0, ws.stream>>>(ws.xs[ws.xcur ^ 1], ws.n, ws.d,
@@ -927,6 +954,7 @@ int eggsync_ctx_pack_owned(eggsync_ctx* ctx, int32_t rank, int32_t ranks, float*
 
 int eggsync_ctx_unpack_owned(eggsync_ctx* ctx, const float* gathered, int32_t ranks) {
   if (!ctx || !gathered || ranks < 1) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
   Workspace& ws = ctx->ws;
   const int64_t cnt = owned_count(ws, ranks), tot = (int64_t)ranks * ws.d * cnt;
   k_unpack_owned<<<(unsigned)((tot + 255) / 256), 256, 0, ws.stream>>>(gathered, ws.n, ws.d, owned_block_points(ws),

@@ -6,12 +6,20 @@ deterministic: Morton keys, stable sort, integer summaries), updates only the
 points it owns (Eq.1 is a Jacobi update, L68, so owned sets are independent
 given D^t), then the ranks exchange their updated points with one all-gather
 (NCCL over NVLink via torch.distributed) and AND-reduce the two criterion
-flags.  The result is bitwise identical to one GPU.
+flags.  The update kernel (tensor-core or SIMT) is chosen from plan statistics
+summed over all ranks (``eggsync_ctx_plan`` + all-reduce +
+``eggsync_ctx_update_planned``), i.e. exactly as one GPU chooses it, and every
+128-point tile is computed the same way on any rank: the result is bitwise
+identical to one GPU.
 
-Ownership is block-interleaved by default: the update's 64-point blocks of the
-sorted order are dealt round-robin to the ranks, so dense cluster cores and
-sparse noise are spread evenly (a contiguous split gives one rank the dense
-core).  torch.distributed is plumbing only; all arithmetic is in the library.
+Ownership is block-interleaved by default: the update's 128-point blocks (the
+tensor-core point tile) of the sorted order are dealt round-robin to the
+ranks, so dense cluster cores and sparse noise are spread evenly (a contiguous
+split gives one rank the dense core).  torch.distributed is plumbing only; all
+arithmetic is in the library.
+
+Streams: the library runs on the context's stream, the collectives on torch's
+current stream; ``TorchComm`` orders them with explicit stream waits.
 """
 from __future__ import annotations
 
@@ -45,7 +53,8 @@ class TorchComm:
     def __init__(self, n: int, d: int, device, group=None, mode: str = "interleaved", ctx=None):
         import torch
         import torch.distributed as dist
-        self.dist, self.group, self.mode = dist, group, mode
+        self.torch, self.dist, self.group, self.mode = torch, dist, group, mode
+        self.device = torch.device(device)
         self.world = dist.get_world_size(group)
         self.rank = dist.get_rank(group)
         span = math.ceil(n / self.world)
@@ -76,11 +85,20 @@ class TorchComm:
             ctx.update(self.lo, self.hi)
 
     def exchange(self, ctx) -> None:
+        torch = self.torch
+        cuda = self.device.type == "cuda"
+        if cuda:
+            xs = torch.cuda.ExternalStream(ctx.stream(), device=self.device)  # the library's stream
+            cs = torch.cuda.current_stream(self.device)                        # the collective's stream
         if self.mode == "interleaved":
             ctx.pack_owned_into(self.rank, self.world, self.send)
         else:
             ctx.pack_into(self.lo, self.cnt, self.send)
+        if cuda:
+            cs.wait_stream(xs)   # the all-gather reads `send` after the pack kernel
         self.dist.all_gather_into_tensor(self.recv, self.send, group=self.group)
+        if cuda:
+            xs.wait_stream(cs)   # the unpack kernel reads `recv` after the all-gather
         view = self.recv.view(self.world, -1, self.cnt)
         if self.mode == "interleaved":
             ctx.unpack_owned_from(view, self.world)

@@ -129,6 +129,17 @@ def _is_torch_cuda(x):
     return type(x).__module__.startswith("torch") and getattr(x, "is_cuda", False)
 
 
+#: cudaStreamLegacy: the legacy default stream as an explicit handle (a NULL handle would
+#: ask the library for its own non-blocking stream, unordered with the caller's work)
+_STREAM_LEGACY = 1
+
+
+def _stream_arg(handle: int):
+    """A torch stream handle for the C ABI: torch's default stream (0) becomes cudaStreamLegacy,
+    so the library's work is ordered after the kernels / copies that produced the tensors."""
+    return ctypes.c_void_p(int(handle) or _STREAM_LEGACY)
+
+
 def _ptr(a):
     if _is_torch_cuda(a):
         return ctypes.c_void_p(a.data_ptr())
@@ -168,7 +179,7 @@ def cluster(points, eps: float, *, max_iters: int = 10000, coords: bool = False,
         n, d = points.shape
         o.device_pointers = 1
         o.device = points.device.index
-        o.stream = ctypes.c_void_p(stream if stream is not None else torch.cuda.current_stream(points.device).cuda_stream)
+        o.stream = _stream_arg(stream if stream is not None else torch.cuda.current_stream(points.device).cuda_stream)
         labels = torch.empty(n, dtype=torch.int32, device=points.device)
         co = torch.empty((n, d), dtype=torch.float32, device=points.device) if coords else None
     else:
@@ -287,6 +298,11 @@ class Context:
         on_dev = _is_torch_cuda(points)
         if not on_dev:
             points = _host_points(points)
+        else:
+            # order the context's stream after the work that produced the tensor
+            import torch
+            torch.cuda.ExternalStream(self.stream(), device=points.device).wait_stream(
+                torch.cuda.current_stream(points.device))
         self._keep = points
         _check(lib().eggsync_ctx_load(self.h, _ptr(points), int(on_dev)))
 
