@@ -246,6 +246,20 @@ int64_t eggsync_ctx_owned_count(eggsync_ctx *ctx, int32_t ranks);
 int eggsync_ctx_pack_owned(eggsync_ctx *ctx, int32_t rank, int32_t ranks, float *buf);
 int eggsync_ctx_unpack_owned(eggsync_ctx *ctx, const float *gathered, int32_t ranks);
 
+/* Collective choice of the update kernel (tensor-core or SIMT) for a multi-rank update, so
+ * that every rank -- and one GPU running the whole range -- choose alike and the result stays
+ * bitwise identical to one GPU.  eggsync_ctx_plan_owned runs the tensor-core plan pass
+ * (Alg 3's neighbour-cell enumeration, L248) for the owned tiles only and writes six host
+ * int64 statistics to stats_out: [0] entries, [1] points in entries, [2] owned tiles,
+ * [3] plan overflow (0/1), [4] largest cell count, [5] tensor cores enabled (0/1).  The
+ * caller reduces them over the ranks -- SUM of [0..2], MAX of [3..5] -- and passes the
+ * result to eggsync_ctx_update_planned, which chooses from the global statistics and runs
+ * the update of the owned tiles (reusing the plan).  Between the two calls nothing else may
+ * run on the context.  Synchronous (the plan statistics are read back to the host).
+ * Errors: EINVAL (bad rank / ranks, no build, NULL stats); ECUDA. */
+int eggsync_ctx_plan_owned(eggsync_ctx *ctx, int32_t rank, int32_t ranks, int64_t *stats_out);
+int eggsync_ctx_update_planned(eggsync_ctx *ctx, int32_t rank, int32_t ranks, const int64_t *global_stats);
+
 /* ------------------------------------------------------------------------
  * Direct SynC (GPU-SynC-style) cross-check and the cluster order parameter
  * (SURVEY.md §8(f) F4).  No grid, no Eq.5 identity: every point is tested

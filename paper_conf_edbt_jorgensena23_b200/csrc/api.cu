@@ -256,6 +256,7 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st, do
       {(void**)&c_cnt, sizeof(int32_t) * cap},
       {(void**)&c_rec, sizeof(float) * CREC * cap},
       {(void**)&c_dig, d <= kTcMaxD ? (size_t)(((kDigMax * (2 * d + 1)) + 15) / 16 * 16) * cap : 0},
+      {(void**)&c_head, d <= kTcMaxD ? sizeof(float) * ceil4(d + 3) * cap : 0},
       {(void**)&c_key, sizeof(uint64_t) * nw * cap},
       {(void**)&t_meta, sizeof(int4) * cap},
       {(void**)&t_parent, sizeof(int32_t) * cap},
@@ -340,10 +341,10 @@ void Workspace::release() {
   }
   buf_give(cur_device, 0, tc_ranges, tc_rcap * sizeof(int2));
   buf_give(cur_device, 1, tc_ent, tc_ecap * sizeof(int32_t));
-  tc_ranges = nullptr;
-  tc_rcap = 0;
   tc_ent = nullptr;
   tc_ecap = 0;
+  tc_ranges = nullptr;
+  tc_rcap = 0;
   for (auto& e : tc_ev)
     if (e) {
       cudaEventDestroy(e);
@@ -932,6 +933,45 @@ int eggsync_ctx_update_owned(eggsync_ctx* ctx, int32_t rank, int32_t ranks) {
   const int rc = stage_update(ctx->ws, 0, ctx->ws.n, nullptr);
   ctx->ws.own_stride = 1;
   ctx->ws.own_offset = 0;
+  return rc;
+}
+
+int eggsync_ctx_plan_owned(eggsync_ctx* ctx, int32_t rank, int32_t ranks, int64_t* stats_out) {
+  if (!ctx || !stats_out || ranks < 1 || rank < 0 || rank >= ranks) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
+  Workspace& ws = ctx->ws;
+  if (!ws.built) {
+    set_error("eggsync_ctx_plan_owned before eggsync_ctx_build");
+    return EGGSYNC_EINVAL;
+  }
+  ws.own_stride = ranks;
+  ws.own_offset = rank;
+  ws.tc_mode = 1;
+  const int rc = stage_update(ws, 0, ws.n, nullptr);
+  ws.tc_mode = 0;
+  ws.own_stride = 1;
+  ws.own_offset = 0;
+  if (rc != EGGSYNC_OK) return rc;
+  for (int k = 0; k < 6; ++k) stats_out[k] = ws.tc_local[k];
+  return EGGSYNC_OK;
+}
+
+int eggsync_ctx_update_planned(eggsync_ctx* ctx, int32_t rank, int32_t ranks, const int64_t* global_stats) {
+  if (!ctx || !global_stats || ranks < 1 || rank < 0 || rank >= ranks) return EGGSYNC_EINVAL;
+  CTX_DEVICE(ctx);
+  Workspace& ws = ctx->ws;
+  if (!ws.built) {
+    set_error("eggsync_ctx_update_planned before eggsync_ctx_build");
+    return EGGSYNC_EINVAL;
+  }
+  for (int k = 0; k < 6; ++k) ws.tc_global[k] = global_stats[k];
+  ws.own_stride = ranks;
+  ws.own_offset = rank;
+  ws.tc_mode = 2;
+  const int rc = stage_update(ws, 0, ws.n, nullptr);
+  ws.tc_mode = 0;
+  ws.own_stride = 1;
+  ws.own_offset = 0;
   return rc;
 }
 

@@ -35,6 +35,23 @@ struct CellRec {
   static constexpr int kFloats = ceil4(3 * D + 3);
 };
 
+// Tensor-core update (update_tc.cuh): per-cell Eq.5 summary as exact integers for the int8
+// GEMM (tcgen05 kind::i8):  v_j = round(sum sin/cos(q_i) * 2^kDigF) (j < 2D), v_2D = count,
+// each in kDigMax balanced base-256 digits; digit column k*(2D+1)+j of a cell's kBytes-byte
+// row.  Stored block-major, c_dig[kBytes/16][cap][16], so that a run of consecutive cells is
+// one contiguous bulk copy per 16-column block (the MN-major GEMM operand layout).  Exact
+// integer accumulation makes the masked sums order-independent.
+// Record head (c_head[kHead/4][cap][4] floats, block-major as well): centre (D), radius,
+// count, start -- a warp reading 32 consecutive cells reads 512 contiguous bytes per block.
+constexpr int kTcMaxD = 12;
+constexpr int kDigF = 21;    // fixed-point bits of the summaries (error <= 2^-22 per cell)
+constexpr int kDigMax = 6;   // |v| <= n * 2^21 < 0.498 * 2^48 for n < 2^24
+template <int D>
+struct CellDig {
+  static constexpr int kBytes = ((kDigMax * (2 * D + 1)) + 15) / 16 * 16;
+  static constexpr int kHead = ((D + 3) + 3) / 4 * 4;  // floats of the record head
+};
+
 // Per-warp staged cell layout in shared memory (floats):
 //   A: c'_0..c'_{D-1}, cc, lim_full, lim_out        (ceil4(D+3))
 //   B: ssin_0..ssin_{D-1}, scos_0..scos_{D-1}       (ceil4(2D))
@@ -184,6 +201,8 @@ struct Workspace {
   uint32_t* c_hi = nullptr;
   int32_t* c_cnt = nullptr;    // [cap]
   float* c_rec = nullptr;      // [cap][CellRec<D>::kFloats]
+  int8_t* c_dig = nullptr;     // [CellDig<D>::kBytes/16][cap][16] (d <= kTcMaxD only)
+  float* c_head = nullptr;     // [CellDig<D>::kHead/4][cap][4] (d <= kTcMaxD only)
   uint64_t* c_key = nullptr;   // [nw][cap]
   // tree (Karras radix tree over sorted cell keys; internal nodes 0..nc-2)
   int4* t_meta = nullptr;      // first, last, left, right
@@ -226,17 +245,23 @@ struct Workspace {
   int32_t* tc_nr = nullptr;     // [tiles+1] ranges per point tile
   int32_t* tc_ne = nullptr;     // [tiles+1] entries per point tile
   int32_t* tc_chunks = nullptr; // [tiles][kChunkMax] first range of each chunk of a tile's range list
-  int32_t* tc_ctr = nullptr;    // [8] ranges allocated, chunk-table overflow, entries (u64), points in entries (u64)
   int32_t* tc_epad = nullptr;   // [tiles+1] entries per tile padded to whole entry tiles
-  int32_t* tc_eoff = nullptr;   // [tiles+1] first entry of each tile in tc_ent (exclusive scan)
+  int32_t* tc_eoff = nullptr;   // [tiles+1] first slot of each tile in tc_ent (exclusive scan)
   int32_t* tc_ent = nullptr;    // unit (cell) of every entry slot, -1 = padding (grown on demand)
+  size_t tc_ecap = 0;
+  int32_t* tc_ctr = nullptr;    // [8] ranges allocated, chunk-table overflow, entries (u64), points in entries (u64), padded entries (u64)
   int32_t* tc_pv = nullptr;     // [tiles] tile index (sort values)
   int32_t* tc_pk = nullptr;     // [tiles] entries, sorted descending (sort keys out)
   int32_t* tc_perm = nullptr;   // [tiles] launch order of the point tiles: most entries first
-  size_t tc_ecap = 0;
   int2* tc_ranges = nullptr;    // (first unit, count), grown on demand (process cache)
   size_t tc_rcap = 0;
   int tc_used = 0;              // 1 when the last update ran on the tensor cores
+  // multi-rank kernel choice (eggsync_ctx_plan_owned / _update_planned): 0 = plan + choose +
+  // run, 1 = plan only (stats into tc_local), 2 = choose from tc_global and run the plan of mode 1
+  int tc_mode = 0;
+  long long tc_local[6] = {0, 0, 0, 0, 0, 0};   // entries, points in entries, tiles, overflow, max cell, enabled
+  long long tc_global[6] = {0, 0, 0, 0, 0, 0};
+  long long tc_pad = 0;                          // padded entries of the local plan
   // tensor-core work accounting (eggsync_ctx_tc_work): since the last reset
   bool tc_timing = false;
   long long tc_acc[5] = {0, 0, 0, 0, 0};  // launches, pairs (unpadded), pairs (padded), alg FLOPs, kernel ns

@@ -307,14 +307,44 @@ __global__ void __launch_bounds__(256) k_cell_sums(const float* __restrict__ xs,
   }
 }
 
-// Hot-loop record of each cell (see CellRec in common.cuh).
+// Hot-loop record of each cell (see CellRec in common.cuh), and for the tensor-core update
+// (D <= kTcMaxD) the cell's Eq.5 summary as exact integers in balanced base-256 digits
+// (CellDig in common.cuh): v_j = round(sum_{q in cell} sin/cos(q_i) * 2^kDigF) from the exact
+// 2^32 fixed-point sums, v_2D = count.  The largest count goes to flags[5] (digits needed).
 template <int D>
 __global__ void k_cell_finalize(int32_t nc, int64_t cap, const int32_t* __restrict__ cell_start,
                                 const uint64_t* __restrict__ c_fix, const uint32_t* __restrict__ c_lo,
                                 const uint32_t* __restrict__ c_hi, const int32_t* __restrict__ c_cnt,
-                                float* __restrict__ c_rec) {
+                                float* __restrict__ c_rec, int8_t* __restrict__ c_dig, float* __restrict__ c_head,
+                                int32_t* __restrict__ flags) {
   const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (c >= nc) return;
+  if constexpr (D <= kTcMaxD) {
+    if (c_dig) {
+      constexpr int NV = 2 * D + 1, DB = CellDig<D>::kBytes;
+      const int32_t cnt = c_cnt[c];
+      atomicMax(&flags[5], cnt);
+      uint32_t w[DB / 4];
+#pragma unroll
+      for (int k = 0; k < DB / 4; ++k) w[k] = 0u;
+#pragma unroll
+      for (int j = 0; j < NV; ++j) {
+        // round half up of fix * 2^(kDigF-32): arithmetic shift of the two's complement sum
+        long long v = j < 2 * D ? (((long long)c_fix[(int64_t)j * cap + c] + (1ll << (31 - kDigF))) >> (32 - kDigF))
+                                : (long long)cnt;
+#pragma unroll
+        for (int k = 0; k < kDigMax; ++k) {
+          const int dk = (int)(int8_t)(uint8_t)(v & 0xff);  // balanced digit in [-128, 127]
+          v = (v - dk) >> 8;
+          const int b = k * NV + j;
+          w[b >> 2] |= (uint32_t)(uint8_t)dk << (8 * (b & 3));
+        }
+      }
+      uint4* dst = reinterpret_cast<uint4*>(c_dig);
+#pragma unroll
+      for (int k = 0; k < DB / 16; ++k) dst[k * cap + c] = make_uint4(w[4 * k], w[4 * k + 1], w[4 * k + 2], w[4 * k + 3]);
+    }
+  }
   constexpr int R = CellRec<D>::kFloats;
   float* r = c_rec + c * R;
   float r2 = 0.f;
@@ -336,6 +366,17 @@ __global__ void k_cell_finalize(int32_t nc, int64_t cap, const int32_t* __restri
     r[2 * D + 3 + i] = (float)((double)(long long)c_fix[(int64_t)(D + i) * cap + c] * kInvFix);
   }
   for (int q = 3 * D + 3; q < R; ++q) r[q] = 0.f;
+  if constexpr (D <= kTcMaxD) {
+    if (c_head) {  // centre, radius, count, start: the tensor-core update's record heads, block-major
+      constexpr int H = CellDig<D>::kHead;
+      float h[H];
+#pragma unroll
+      for (int q = 0; q < H; ++q) h[q] = q < D + 3 ? r[q] : 0.f;
+      float4* dst = reinterpret_cast<float4*>(c_head);
+#pragma unroll
+      for (int k = 0; k < H / 4; ++k) dst[k * cap + c] = make_float4(h[4 * k], h[4 * k + 1], h[4 * k + 2], h[4 * k + 3]);
+    }
+  }
 }
 
 // ------------------------------------------------------- A5 radix tree (Karras 2012)
@@ -526,6 +567,7 @@ static int build_d(Workspace& ws) {
   k_keys<D><<<blocks_for(n, T), T, 0, st>>>(ws.xs[ws.xcur], n, K.bits, K.sub, K.nw, K.w, K.inv_cw, ws.keys);
   EGG_LAUNCH_CHECK();
   EGG_CUDA(cudaMemsetAsync(ws.flags + 2, 0, sizeof(int32_t), st));
+  EGG_CUDA(cudaMemsetAsync(ws.flags + 5, 0, sizeof(int32_t), st));  // largest cell count (k_cell_finalize)
   if (n > 1) {
     k_check_sorted<<<blocks_for(n - 1, T), T, 0, st>>>(ws.keys, n, K.nw, ws.flags);
     EGG_LAUNCH_CHECK();
@@ -591,7 +633,7 @@ static int build_d(Workspace& ws) {
   ws.n_cells = ws.h_flags[6] + 1;
   const int32_t nc = ws.n_cells;
   k_cell_finalize<D><<<blocks_for(nc, T), T, 0, st>>>(nc, cap, ws.cell_start, ws.c_fix, ws.c_lo, ws.c_hi,
-                                                      ws.c_cnt, ws.c_rec);
+                                                      ws.c_cnt, ws.c_rec, ws.c_dig, ws.c_head, ws.flags);
   EGG_LAUNCH_CHECK();
   if (K.sub > 0) {
     ws.n_grid = ws.h_flags[7] + 1;

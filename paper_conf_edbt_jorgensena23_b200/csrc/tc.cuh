@@ -32,6 +32,20 @@ __device__ __forceinline__ void bar_wait(uint64_t* b, uint32_t parity) {
       : "memory");
 }
 
+// wait with a suspend-time hint: the thread sleeps until the phase completes (or ~1 ms passes)
+// instead of re-polling, so waiting warps give their issue slots to the working ones
+__device__ __forceinline__ void bar_sleep(uint64_t* b, uint32_t parity) {
+#ifdef EGG_TC_SPIN
+  bar_wait(b, parity);
+  return;
+#endif
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, 1000000;\n @!p bra WAIT_%=;\n}" ::"r"(
+          smem_addr(b)),
+      "r"(parity)
+      : "memory");
+}
+
 // ---- TMEM allocation (one warp, power-of-two columns >= 32) -----------------
 template <uint32_t kCols>
 __device__ __forceinline__ void tmem_alloc(uint32_t* dst_smem) {
@@ -73,6 +87,24 @@ __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t
 __host__ __device__ constexpr uint32_t idesc_tf32(int M, int N, bool b_mn_major) {
   return (1u << 4) | (2u << 7) | (2u << 10) | ((b_mn_major ? 1u : 0u) << 16) | ((uint32_t)(N >> 3) << 17) |
          ((uint32_t)(M >> 4) << 24);
+}
+
+// ---- instruction descriptor: kind::i8, signed 8-bit A and B, s32 accumulate ----
+//  bits [4,6) D format (2 = S32), [7,10) A format (1 = signed 8-bit), [10,13) B format,
+//  bit 16 B major (1 = MN), [17,23) N>>3, [24,29) M>>4
+__host__ __device__ constexpr uint32_t idesc_s8(int M, int N, bool b_mn_major) {
+  return (2u << 4) | (1u << 7) | (1u << 10) | ((b_mn_major ? 1u : 0u) << 16) | ((uint32_t)(N >> 3) << 17) |
+         ((uint32_t)(M >> 4) << 24);
+}
+
+// D[tmem] (+)= A[tmem] * B[smem]^T, int8 x int8 -> int32 (A: M x 32 int8 = 8 TMEM columns)
+__device__ __forceinline__ void mma_ts_s8(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
+                                          uint32_t accumulate) {
+  asm volatile(
+      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+      " tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n}" ::"r"(d_tmem),
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
+      : "memory");
 }
 
 // D[tmem] (+)= A[tmem] * B[smem]^T  (A: M x 8 tf32 columns of TMEM, one row per lane)
@@ -117,6 +149,14 @@ __device__ __forceinline__ void st32(uint32_t taddr, const uint32_t (&v)[32]) {
       "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15]), "r"(v[16]), "r"(v[17]), "r"(v[18]),
       "r"(v[19]), "r"(v[20]), "r"(v[21]), "r"(v[22]), "r"(v[23]), "r"(v[24]), "r"(v[25]), "r"(v[26]), "r"(v[27]),
       "r"(v[28]), "r"(v[29]), "r"(v[30]), "r"(v[31])
+      : "memory");
+}
+__device__ __forceinline__ void st16(uint32_t taddr, const uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+          taddr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]), "r"(v[9]),
+      "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
       : "memory");
 }
 __device__ __forceinline__ void st8(uint32_t taddr, const uint32_t (&v)[8]) {

@@ -6,34 +6,39 @@
 // are computed for a tile of 128 consecutive sorted points at a time as two
 // dense contractions against "entries" (update units = cells of the hierarchy):
 //
-//   GEMM1  S[p][e] = -2 q_p . c'_e - L_e        (tf32 x3 split: ~fp32-exact)
+//   GEMM1  S[p][e] = -2 q_p . c'_e - L_e        (kind::tf32, x3 hi/lo split: ~fp32-exact)
 //          v = |q_p|^2 + S = |p - c_e|^2 - limF_e   in the tile-shifted frame
 //   classify (CUDA cores, one thread per point row of TMEM):
-//          v <= 0            -> entry e entirely inside the eps-ball of p (Eq.6 full part)
-//          0 < v <= W_e      -> ambiguous band: exact fp64 re-decision (single point) or
+//          v < 0 (sign bit)  -> entry e entirely inside the eps-ball of p (Eq.6 full part)
+//          0 <= v <= W_e     -> ambiguous band: exact fp64 re-decision (single point) or
 //                               exact scan of the unit's points (Eq.6 partial part)
 //          v > W_e           -> outside
-//          P[p][e] = 1 for "inside", else 0   (written back into TMEM over S)
-//   GEMM2  O[p][:] += P[p][:] . V[:][:]        V_e = (sum sin - cnt sin o, sum cos - cnt cos o, cnt)
-//                                              split hi/lo into tf32 pairs (N = 2(2D+1))
+//          P[p][e] = -1 (int8) for "inside", else 0, written back into TMEM over S
+//   GEMM2  O[p][:] += P[p][:] . V[:][:]        (kind::i8, int32 accumulate: EXACT)
+//          V_e = the unit's summary as integers v = round(sum sin/cos * 2^21) and its count,
+//          each split into balanced base-256 digits (CellDig, built in k_cell_finalize);
+//          N = digits x (2D+1) columns, digits from the largest cell count (3 at C3 iteration 1)
 //
-// with fp32 accumulation in TMEM drained every kDrain entry tiles into exact 64-bit
-// fixed-point sums (2^-32) per classifier group in shared memory.
+// Integer accumulation makes the sums exact and order-independent: no fp32 drain of TMEM,
+// one accumulator for both classifier groups, read once in the epilogue.  P as int8 is a
+// quarter of the TMEM write traffic of an fp32 mask.
 // Entries are the cells of the subtrees that the plan pass (k_tc_plan) could not
 // decide for the whole tile; subtrees entirely inside for every point that still
 // needs them are added per point in the plan pass (full_S / full_N, exact fp64 of
-// the fp32 subtree sums, as in k_update).  k_tc_expand turns each tile's ranges into a
-// slot list (one unit per entry, padded to whole entry tiles); tiles are launched
-// heaviest-first.
+// the fp32 subtree sums, as in k_update).  k_tc_expand turns each tile's ranges into a slot
+// list (one unit per entry, padded to whole entry tiles); tiles are launched heaviest-first.
 //
-// Roles (416 threads, one CTA per point tile, one CTA per SM: it owns all 512 TMEM columns):
+// Roles (448 threads, one CTA per point tile, one CTA per SM: it owns all 512 TMEM columns):
 //   warps 0-3   classifier group 0 (TMEM lanes 0..127), even entry tiles
 //   warps 4-7   classifier group 1, odd entry tiles
-//   warps 8-11  producers: thread t owns entry slot t; stages the unit record with
-//               cp.async one tile ahead and writes the GEMM operands (origin-shifted,
-//               tf32-split) into a 3-stage shared-memory ring
-//   warp 12     MMA issue (one thread, polling both GEMM conditions) and TMEM owner
-// TMEM: Q (K1 columns) | 3 S/P buffers (GEMM1 runs up to 2 tiles ahead) | O per group.
+//   warps 8-11  producers: thread t owns entry slot t; copies the unit's record head and
+//               digit row (block-major global layouts: coalesced along runs of units) with
+//               cp.async into the ring stage one tile ahead, then writes the origin-shifted,
+//               tf32-split GEMM1 operand row (ring of up to 8 shared-memory stages)
+//   warp 12     GEMM1 issue (one thread) and TMEM owner
+//   warp 13     GEMM2 issue (one thread): decoupled from GEMM1, so a classifier group
+//               waiting on its P never holds back the next S
+// TMEM: Q (K1 columns) | 2-3 S/P buffers of 128 columns | O (N columns, int32).
 #pragma once
 #include <cub/cub.cuh>
 
@@ -46,52 +51,33 @@ namespace egg {
 
 constexpr int kTcTile = 128;  // points per tile (TMEM lanes, GEMM M)
 constexpr int kTcEnt = 128;   // entries per entry tile (GEMM1 N, GEMM2 K)
-constexpr int kTcThreads = 13 * 32;  // 8 classifier + 4 producer warps + 1 MMA warp (<= 128 registers)
-constexpr int kProd = 128;  // producer threads (warps 8-11): one entry slot each
-constexpr int kMmaWarp = 12;  // TMEM owner; its lane 0 issues the MMAs
-constexpr int kTcMaxD = 12;
-#ifndef EGG_TC_DRAIN
-#define EGG_TC_DRAIN 2
-#endif
-constexpr int kDrain = EGG_TC_DRAIN;  // entry tiles per fp32 chunk of a classifier group
+constexpr int kProdWarps = 4;  // producers: one entry slot per thread
+constexpr int kProd = 32 * kProdWarps;
+constexpr int kMma1Warp = 8 + kProdWarps;  // GEMM1 issue (one thread) + TMEM owner
+constexpr int kMma2Warp = kMma1Warp + 1;   // GEMM2 issue (one thread)
+constexpr int kTcThreads = (kMma2Warp + 1) * 32;  // 8 classifier + 4 producer + 2 MMA warps
+constexpr int kTcMaxStages = 8;
 
 template <int D>
 struct TcCfg {
   static constexpr int K1 = ((3 * D + 2) + 7) / 8 * 8;  // GEMM1 K: q_hi, q_lo, q_hi, 1, 1
   static constexpr int NV = 2 * D + 1;                  // sin, cos, count
-  static constexpr int N2 = (2 * NV + 15) / 16 * 16;     // GEMM2 N: hi | lo
-  // TMEM columns: Q, NS S/P buffers (3 when they fit: GEMM1 runs ahead of both
-  // classifier groups), one O accumulator per classifier group
-  static constexpr int kColQ = 0;
-  static constexpr int kColS = K1;                  // S/P buffers: kColS + 128*b
-#ifndef EGG_TC_NS
-#define EGG_TC_NS 3
-#endif
-  static constexpr int kNS0 = (EGG_TC_NS >= 3 && K1 + 3 * kTcEnt + 2 * N2 <= 512) ? 3 : 2;
-  static constexpr int kColO0 = K1 + kNS0 * kTcEnt;
-  static_assert(K1 + 2 * kTcEnt + 2 * N2 <= 512, "TMEM budget");
-  static_assert(N2 % 16 == 0, "drain loads of 16 columns");
-  // shared-memory stage: B1 (K-major: entry rows), B2 (K-major: value rows), meta
+  static constexpr int DB = CellDig<D>::kBytes;         // digit row of a cell (GEMM2 N <= DB)
+  static constexpr int R = CellRec<D>::kFloats;
+  static constexpr int R0 = CellDig<D>::kHead;          // record head: centre, radius, count, start
+  static constexpr int R0S = (R0 / 4) % 2 == 0 ? R0 + 4 : R0;  // shared stride: conflict-free 16-B accesses
+  static constexpr int kRecBytes = kTcEnt * R0S * 4;   // record heads of a stage's entries (cp.async)
+  // shared memory: ring stages (run-time size, TcStage) | raw record heads | rare sums | misc
   static constexpr int SBO1 = (K1 / 4) * 128;
   static constexpr int kB1Bytes = kTcEnt * K1 * 4;
-  static constexpr int LBO2 = 144;  // 16-byte gap per 4-entry chunk: conflict-free producer stores
-  static constexpr int SBO2 = (kTcEnt / 4) * LBO2;
-  static constexpr int kB2Bytes = (N2 / 8) * SBO2;
-  static constexpr int kMetaBytes = kTcEnt * 16 + 16;  // W, cnt, start, cell; Wmax[4]
-  static constexpr int kStageBytes = kB1Bytes + kB2Bytes + kMetaBytes;
-  static constexpr int R = CellRec<D>::kFloats;
-  static constexpr int kRawBytes = 2 * kTcEnt * R * 4;      // cell records staged by bulk copies [2][128][R]
-  // per classifier group: exact fixed-point sums [NV][row] (rare-path count at 2D) + tensor-core count [row]
-  static constexpr int kRareBytes = 2 * (NV + 1) * kTcTile * 8;
-  static constexpr int kMiscBytes = 3072;
-  static constexpr int kBudget = 227 * 1024 - 1024;
-  static constexpr int kStages0 = (kBudget - kRawBytes - kRareBytes - kMiscBytes) / kStageBytes;
-  static constexpr int kStages = kStages0 >= 4 ? 4 : (kStages0 >= 3 ? 3 : 2);
-  static constexpr int kRingBytes = kStages * kStageBytes;
-  static constexpr int kNS = kNS0 < kStages ? kNS0 : kStages;  // the MMA loop needs stages >= S buffers
-  static constexpr int kColO = K1 + kNS * kTcEnt;   // O buffers: kColO + N2*g
-  static constexpr size_t kSmem = (size_t)kRingBytes + kRawBytes + kRareBytes + kMiscBytes + 1024;  // +1024 align
-  static_assert(kSmem <= 227 * 1024, "shared-memory budget");
+  static constexpr int kRareBytes = NV * kTcTile * 8;   // exact sums [2D][row] (2^-32) + count [row]
+  static constexpr int kSlotBytes = 4 * kTcEnt * 4;     // slot units of 4 entry tiles (producers' ring)
+  static constexpr int kMiscBytes = 1024;
+  static constexpr int kFixedBytes = kRareBytes + kSlotBytes + kMiscBytes + 1024;  // +1024 alignment
+  static constexpr int kBudget = 227 * 1024;
+  __host__ __device__ static constexpr int stage_bytes(int n2) {
+    return (kB1Bytes + n2 * kTcEnt + kRecBytes + 8 * kTcEnt + 16 + 127) / 128 * 128;
+  }
 };
 
 // ----------------------------------------------------------------------------------------
@@ -118,10 +104,10 @@ struct PlanArgs {
   float e;
   int32_t* t_nr;              // [ntiles] ranges per tile
   int32_t* t_ne;              // [ntiles] entries per tile
-  int32_t* t_epad;            // [ntiles] entries padded to whole entry tiles
   int32_t* t_pv;              // [ntiles] tile index (values of the launch-order sort)
   int32_t* chunks;            // [ntiles][kChunkMax] first slot of each chunk
-  int32_t* ctr;               // [0] slots allocated, [1] chunk-table overflow, [2..3] entries (u64), [4..5] their points (u64)
+  int32_t* t_epad;            // [ntiles] entries padded to whole entry tiles (scan -> slot offsets)
+  int32_t* ctr;               // [0] slots allocated, [1] chunk-table overflow, [2..3] entries (u64), [4..5] their points (u64), [6..7] entries padded to whole entry tiles (u64)
   int64_t rcap;               // capacity of ranges
   int2* ranges;               // (first cell, count)
   double* full_S;             // [2D][n]
@@ -313,6 +299,7 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
     a.t_ne[tile] = ne;
     atomicAdd(reinterpret_cast<unsigned long long*>(a.ctr + 2), (unsigned long long)ne);  // unpadded entries
     atomicAdd(reinterpret_cast<unsigned long long*>(a.ctr + 4), (unsigned long long)npts);
+    atomicAdd(reinterpret_cast<unsigned long long*>(a.ctr + 6), (unsigned long long)((ne + kTcEnt - 1) / kTcEnt * kTcEnt));
     a.t_epad[tile] = (ne + kTcEnt - 1) / kTcEnt * kTcEnt;
     a.t_pv[tile] = (int32_t)tile;
   }
@@ -378,33 +365,38 @@ struct TcArgs {
   const int32_t* __restrict__ g_of;
   const int32_t* __restrict__ g_cnt;
   const float* __restrict__ c_rec;
+  const int8_t* __restrict__ c_dig;   // [DB/16][cap][16] block-major digit rows
+  const float* __restrict__ c_head;   // [cap][R0] record heads
+  const int32_t* __restrict__ cell_of;  // unit of each sorted point
   const uint32_t* __restrict__ c_lo;
   const uint32_t* __restrict__ c_hi;
-  const int32_t* __restrict__ ent;   // unit of every entry slot (-1 = padding)
-  const int32_t* __restrict__ eoff;  // [ntiles] first slot of each point tile
-  const int32_t* __restrict__ perm;  // [ntiles] launch order
+  const int32_t* __restrict__ ent;    // unit of every entry slot (-1 = padding), k_tc_expand
+  const int32_t* __restrict__ eoff;   // [ntiles] first slot of each point tile
+  const int32_t* __restrict__ perm;   // [ntiles] launch order
   const int32_t* __restrict__ t_ne;
   const double* __restrict__ full_S;
   const int32_t* __restrict__ full_N;
   int64_t n, cap, lo, hi;
   int32_t ntiles, stride, offset;
+  int32_t ndig, n2, nst, ns;   // digits per value, GEMM2 N, ring stages, S buffers (run-time layout)
+  int32_t stage_bytes;
   float e, e2f, rel;
   double e2d;
   int32_t* flags;
   int32_t* nbr;
-  unsigned long long* prof;  // optional cycle accounting (EGGSYNC_TC_PROF)
+  unsigned long long* prof;  // EGG_TC_PROF builds: [16] cycle sums
 };
-
 
 // shared-memory header of the TC kernel
 struct TcMisc {
-  uint64_t stage_full[4], stage_empty[4], s_full[3], p_full[3], o_full[2];  // s_full / p_full: per S buffer
+  uint64_t stage_full[kTcMaxStages], stage_empty[kTcMaxStages];
+  uint64_t s_full[3], p_full[3], s_free[3], o_done;
   uint32_t tbase;
-  float o[kTcMaxD], s0[kTcMaxD], c0[kTcMaxD];
+  float o[kTcMaxD];
   float lo[4][kTcMaxD], hi[4][kTcMaxD];
   float Rq, Rqi;
 };
-static_assert(sizeof(TcMisc) <= 3072, "misc header");
+static_assert(sizeof(TcMisc) <= 1024, "misc header");
 
 // per-thread asynchronous 16-byte global -> shared copies (L2 only), waited per thread
 __device__ __forceinline__ void cp_async16(void* dst, const void* src) {
@@ -416,42 +408,54 @@ __device__ __forceinline__ void cp_async_wait() {
   asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
 }
 
+// One ring stage (run-time size: GEMM2 N = n2 depends on the digits needed):
+//   b1   [kTcEnt][K1] tf32, K-major core matrices (GEMM1 B: entry rows)            (producers)
+//   b2   [n2/16][kTcEnt][16] int8, MN-major core matrices (GEMM2 B: digits x entries) (cp.async)
+//   rec  [kTcEnt][R0S] record heads: centre (= the point of a singleton), radius, count, start (cp.async)
+//   W, cell [kTcEnt] band width and unit of every slot (-1 = padding); wmax[4]       (producers)
 template <int D>
 struct TcStage {
   float* b1;
-  float* b2;
+  int8_t* b2;
+  float* rec;
   float* W;
-  int32_t* cnt;
-  int32_t* start;
   int32_t* cell;
   float* wmax;
-  __device__ TcStage(unsigned char* ring, int s) {
+  __device__ TcStage(unsigned char* ring, int s, int stage_bytes, int n2) {
     using C = TcCfg<D>;
-    unsigned char* p = ring + (size_t)s * C::kStageBytes;
+    unsigned char* p = ring + (size_t)s * stage_bytes;
     b1 = reinterpret_cast<float*>(p);
-    b2 = reinterpret_cast<float*>(p + C::kB1Bytes);
-    unsigned char* m = p + C::kB1Bytes + C::kB2Bytes;
+    b2 = reinterpret_cast<int8_t*>(p + C::kB1Bytes);
+    rec = reinterpret_cast<float*>(p + C::kB1Bytes + n2 * kTcEnt);
+    unsigned char* m = p + C::kB1Bytes + n2 * kTcEnt + C::kRecBytes;
     W = reinterpret_cast<float*>(m);
-    cnt = reinterpret_cast<int32_t*>(m + 4 * kTcEnt);
-    start = reinterpret_cast<int32_t*>(m + 8 * kTcEnt);
-    cell = reinterpret_cast<int32_t*>(m + 12 * kTcEnt);
-    wmax = reinterpret_cast<float*>(m + 16 * kTcEnt);
+    cell = reinterpret_cast<int32_t*>(m + 4 * kTcEnt);
+    wmax = reinterpret_cast<float*>(m + 8 * kTcEnt);
   }
+  __device__ int32_t cnt(int e) const { return __float_as_int(rec[e * TcCfg<D>::R0S + D + 1]); }
+  __device__ int32_t start(int e) const { return __float_as_int(rec[e * TcCfg<D>::R0S + D + 2]); }
+  __device__ float pt(int e, int i) const { return rec[e * TcCfg<D>::R0S + i]; }
 };
+
+// record head field i (centre 0..D-1, radius D, count D+1, start D+2) of unit c (block-major)
+template <int D>
+__device__ __forceinline__ float head_f(const float* __restrict__ c_head, int64_t cap, int32_t c, int i) {
+  return c_head[((int64_t)(i >> 2) * cap + c) * 4 + (i & 3)];
+}
 
 // Exact path for a multi-point unit e inside the band of point pe (P stays 0 for the pair):
 // refine with the unit's exact MBR, then its points one by one (fp32 + fp64 re-decision as
-// in k_update).  Sums go into the classifier group's own fixed-point (2^-32) sums [NV][row]:
-// exact, and the two groups' arrays are added in the epilogue (order-independent).
+// in k_update).  Sums go into the row's exact fixed-point (2^-32) sums in shared memory
+// (64-bit shared atomics: both classifier groups may add to the same row).
 __device__ __forceinline__ void rare_add(unsigned long long* rare, int i, int row, double v) {
-  rare[i * kTcTile + row] += (unsigned long long)llrint(v * kFix);  // the group's own row: no atomics
+  atomicAdd(&rare[i * kTcTile + row], (unsigned long long)llrint(v * kFix));
 }
 template <int D>
-__device__ __noinline__ void tc_rare(const TcArgs<D>& a, const float* __restrict__ pe, int e,
+__device__ __forceinline__ void tc_rare(const TcArgs<D>& a, const float* __restrict__ pe, int e,
                                      const TcStage<D>& st, unsigned long long* __restrict__ rare, int row) {
-  const int32_t cnt = st.cnt[e];
-  const int32_t start = st.start[e];
   const int32_t c = st.cell[e];
+  const int32_t cnt = st.cnt(e);
+  const int32_t start = st.start(e);
   float mind = 0.f, maxd = 0.f;
 #pragma unroll
   for (int i = 0; i < D; ++i) {
@@ -463,14 +467,6 @@ __device__ __noinline__ void tc_rare(const TcArgs<D>& a, const float* __restrict
   }
   const float lim_in = a.e2f * (1.f - a.rel), lim_out = a.e2f * (1.f + a.rel);
   if (mind > lim_out) return;
-  constexpr int R = CellRec<D>::kFloats;
-  if (maxd <= lim_in) {  // the whole unit is inside: its summary
-    const float* __restrict__ r = a.c_rec + (int64_t)c * R;
-#pragma unroll
-    for (int i = 0; i < 2 * D; ++i) rare_add(rare, i, row, (double)r[D + 3 + i]);
-    rare[2 * D * kTcTile + row] += (unsigned long long)cnt;
-    return;
-  }
   unsigned long long nin = 0;
   for (int32_t t = 0; t < cnt; ++t) {
     const int64_t qi = start + t;
@@ -482,7 +478,7 @@ __device__ __noinline__ void tc_rare(const TcArgs<D>& a, const float* __restrict
       const float u = qv[i] - pe[i];
       d2 = fmaf(u, u, d2);
     }
-    bool in = d2 <= lim_in;
+    bool in = maxd <= lim_in || d2 <= lim_in;
     if (!in && d2 <= lim_out) in = exact_d2<D>(qv, pe) <= a.e2d;
     if (in) {
 #pragma unroll
@@ -493,26 +489,24 @@ __device__ __noinline__ void tc_rare(const TcArgs<D>& a, const float* __restrict
       ++nin;
     }
   }
-  rare[2 * D * kTcTile + row] += nin;
+  if (nin) atomicAdd(&rare[2 * D * kTcTile + row], nin);
 }
 
-// Build entry slot `pt` (unit c, or padding when c < 0) of a stage: B1 row, B2 column, meta.
+// Build entry slot `pt` (unit c, or padding when c < 0) of a stage: B1 row and metadata from
+// the unit's record head (prefetched into registers); its digit row (B2) came by cp.async.
 template <int D>
 __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const TcMisc* __restrict__ ms,
                                                 const TcStage<D>& st, int pt, int32_t c,
                                                 const float* __restrict__ rec, float Rq, float Rqi) {
   using C = TcCfg<D>;
-  constexpr int K1 = C::K1, NV = C::NV, N2 = C::N2;
-  constexpr int R = CellRec<D>::kFloats;
+  constexpr int K1 = C::K1;
   float b[K1];
-  float vh[NV], vl[NV];
   float W = 0.f;
-  int32_t ccnt = 0, cstart = 0;
   if (c >= 0) {
-    float r[R];
-    const float4* r4 = reinterpret_cast<const float4*>(rec);  // staged by the bulk copy
+    float r[C::R0];
+    const float4* r4 = reinterpret_cast<const float4*>(rec);  // staged by cp.async
 #pragma unroll
-    for (int k = 0; k < R / 4; ++k) {
+    for (int k = 0; k < C::R0 / 4; ++k) {
       const float4 t4 = r4[k];
       r[4 * k] = t4.x;
       r[4 * k + 1] = t4.y;
@@ -531,8 +525,6 @@ __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const TcMisc
       cinf = fmaxf(cinf, fabsf(cp));
     }
     const float rad = r[D];
-    ccnt = __float_as_int(r[D + 1]);
-    cstart = __float_as_int(r[D + 2]);
     // error budget: eta = rounding of the shifted frame; E = tf32 split
     // (2^-17 |q||c'|) + tensor-core accumulation (4 K-steps x 9 terms x 2^-23 of the sum
     // of |terms| <= 2^-17.8 (2|q||c'| + |L|)) + fp32 |q|^2, |c'|^2, L and v roundings
@@ -548,27 +540,10 @@ __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const TcMisc
     const float Lh = tc::tf32_hi(L);
     b[3 * D] = -Lh;
     b[3 * D + 1] = -(L - Lh);
-    const float fc = (float)ccnt;
-#pragma unroll
-    for (int i = 0; i < D; ++i) {
-      const float vs = fmaf(-fc, ms->s0[i], r[D + 3 + i]);
-      const float vc = fmaf(-fc, ms->c0[i], r[2 * D + 3 + i]);
-      vh[i] = tc::tf32_hi(vs);
-      vl[i] = vs - vh[i];
-      vh[D + i] = tc::tf32_hi(vc);
-      vl[D + i] = vc - vh[D + i];
-    }
-    vh[2 * D] = tc::tf32_hi(fc);
-    vl[2 * D] = fc - vh[2 * D];
   } else {
 #pragma unroll
     for (int k = 0; k < 3 * D + 2; ++k) b[k] = 0.f;
     b[3 * D] = 1073741824.f;  // v = 2^30: outside, never ambiguous
-#pragma unroll
-#pragma unroll
-    for (int k = 0; k < NV; ++k) vh[k] = vl[k] = 0.f;
-    ccnt = 0;
-    cstart = 0;
   }
 #pragma unroll
   for (int k = 3 * D + 2; k < K1; ++k) b[k] = 0.f;
@@ -579,41 +554,66 @@ __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const TcMisc
     for (int kc = 0; kc < K1 / 4; ++kc)
       *reinterpret_cast<float4*>(b1 + kc * 128) = make_float4(b[4 * kc], b[4 * kc + 1], b[4 * kc + 2], b[4 * kc + 3]);
   }
-  // B2: K-major value rows n (hi: n < NV, lo: NV <= n < 2NV), entry columns
-  {
-    unsigned char* b2 = reinterpret_cast<unsigned char*>(st.b2) + (pt >> 2) * C::LBO2 + (pt & 3) * 4;
-#pragma unroll
-    for (int n = 0; n < NV; ++n) {
-      *reinterpret_cast<float*>(b2 + (n >> 3) * C::SBO2 + (n & 7) * 16) = vh[n];
-      const int n2 = NV + n;
-      *reinterpret_cast<float*>(b2 + (n2 >> 3) * C::SBO2 + (n2 & 7) * 16) = vl[n];
-    }
-#pragma unroll
-    for (int n = 2 * NV; n < N2; ++n) *reinterpret_cast<float*>(b2 + (n >> 3) * C::SBO2 + (n & 7) * 16) = 0.f;
-  }
-#pragma unroll
-  st.cnt[pt] = ccnt;
-  st.start[pt] = cstart;
-  st.cell[pt] = c;
+  st.W[pt] = W;
   return W;
 }
 
+// Development-only cycle accounting (-DEGG_TC_PROF): per-role waits / work summed over CTAs
+#ifdef EGG_TC_PROF
+#define TCP_T(v) const long long v = clock64()
+#define TCP_ADD(k, d) prof_acc[k] += (unsigned long long)(d)
+#else
+#define TCP_T(v)
+#define TCP_ADD(k, d)
+#endif
+
+// (t % n, (t / n) & 1) of a ring position t, maintained incrementally (no integer division)
+struct RingPos {
+  int i = 0;
+  uint32_t ph = 0;
+  __device__ __forceinline__ void adv(int n) {
+    if (++i == n) {
+      i = 0;
+      ph ^= 1u;
+    }
+  }
+};
+
+// sign bits of four fp32 values -> four int8 mask bytes (0xFF where the value is negative / -0)
+// (prmt's default mode: a selector nibble with bit 3 set replicates the selected byte's sign)
+__device__ __forceinline__ uint32_t prmt(uint32_t a, uint32_t b, uint32_t sel) {
+  uint32_t r;
+  asm("prmt.b32 %0, %1, %2, %3;" : "=r"(r) : "r"(a), "r"(b), "r"(sel));
+  return r;
+}
+__device__ __forceinline__ uint32_t sign_bytes4(uint32_t a, uint32_t b, uint32_t c, uint32_t d) {
+  const uint32_t x = prmt(a, b, 0x00FBu);  // [sgn(a.b3), sgn(b.b3), ., .]
+  const uint32_t y = prmt(c, d, 0x00FBu);
+  return prmt(x, y, 0x5410u);
+}
+
 template <int D>
-__global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) {
+// registers: warps are dealt round-robin to the 4 SM sub-partitions (16K registers each)
+__global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc(const TcArgs<D> a) {
   using C = TcCfg<D>;
-  constexpr int K1 = C::K1, NV = C::NV, N2 = C::N2, NST = C::kStages;
+  constexpr int K1 = C::K1, NV = C::NV, R0 = C::R0;
   extern __shared__ __align__(16) unsigned char tsm_raw[];
   unsigned char* tsm = tsm_raw + ((1024u - (tc::smem_addr(tsm_raw) & 1023u)) & 1023u);
+  const int NST = a.nst, NS = a.ns, SB = a.stage_bytes, N2 = a.n2;
   unsigned char* ring = tsm;
-  float* raw = reinterpret_cast<float*>(tsm + C::kRingBytes);  // [2][kTcEnt][R] staged cell records
-  unsigned long long* rare = reinterpret_cast<unsigned long long*>(tsm + C::kRingBytes + C::kRawBytes);
-  TcMisc* ms = reinterpret_cast<TcMisc*>(tsm + C::kRingBytes + C::kRawBytes + C::kRareBytes);
+  unsigned long long* rare = reinterpret_cast<unsigned long long*>(tsm + (size_t)NST * SB);
+  int32_t* slots = reinterpret_cast<int32_t*>(tsm + (size_t)NST * SB + C::kRareBytes);
+  TcMisc* ms = reinterpret_cast<TcMisc*>(tsm + (size_t)NST * SB + C::kRareBytes + C::kSlotBytes);
 
   const int tid = threadIdx.x, wid = tid >> 5, lane = tid & 31;
   const int64_t tile = a.perm[blockIdx.x];  // heaviest point tiles first (shorter tail)
   const int64_t base = tc_tile_base(a.lo, tile, a.stride, a.offset);
   const int32_t ne = a.t_ne[tile];
   const int T = (ne + kTcEnt - 1) / kTcEnt;  // entry tiles (the slot list is padded to T * kTcEnt)
+  const int kColS = K1, kColO = K1 + NS * kTcEnt;
+#ifdef EGG_TC_PROF
+  unsigned long long prof_acc[4] = {0, 0, 0, 0};
+#endif
 
   // ---- setup -------------------------------------------------------------------------
   if (tid == 0) {
@@ -621,15 +621,16 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
       tc::bar_init(&ms->stage_full[s], kProd);
       tc::bar_init(&ms->stage_empty[s], 1);
     }
-    for (int b = 0; b < C::kNS; ++b) {
+    for (int b = 0; b < NS; ++b) {
       tc::bar_init(&ms->s_full[b], 1);
       tc::bar_init(&ms->p_full[b], kTcTile);
+      tc::bar_init(&ms->s_free[b], 1);
     }
-    for (int b = 0; b < 2; ++b) tc::bar_init(&ms->o_full[b], 1);
+    tc::bar_init(&ms->o_done, 1);
     tc::bar_fence_init();
   }
-  if (wid == kMmaWarp) tc::tmem_alloc<512>(&ms->tbase);
-  for (int t = tid; t < 2 * (NV + 1) * kTcTile; t += kTcThreads) rare[t] = 0ull;
+  if (wid == kMma1Warp) tc::tmem_alloc<512>(&ms->tbase);
+  for (int t = tid; t < NV * kTcTile; t += kTcThreads) rare[t] = 0ull;
 
   // classifier rows: every classifier thread holds its point
   const bool is_cls = wid < 8;
@@ -659,10 +660,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
   if (tid < D) {
     float l = fminf(fminf(ms->lo[0][tid], ms->lo[1][tid]), fminf(ms->lo[2][tid], ms->lo[3][tid]));
     float h = fmaxf(fmaxf(ms->hi[0][tid], ms->hi[1][tid]), fmaxf(ms->hi[2][tid], ms->hi[3][tid]));
-    const float o = 0.5f * (l + h);
-    ms->o[tid] = o;
-    ms->s0[tid] = sinf(o);
-    ms->c0[tid] = cosf(o);
+    ms->o[tid] = 0.5f * (l + h);
   }
   if (tid == 0) {
     ms->Rq = 0.f;
@@ -704,7 +702,7 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
       v[3 * D + 1] = __float_as_uint(1.f);
 #pragma unroll
       for (int k = 3 * D + 2; k < K1; ++k) v[k] = 0u;
-      const uint32_t taddr = ms->tbase + ((uint32_t)(32 * (wid & 3)) << 16) + C::kColQ;
+      const uint32_t taddr = ms->tbase + ((uint32_t)(32 * (wid & 3)) << 16);
 #pragma unroll
       for (int c = 0; c < K1 / 8; ++c) {
         uint32_t w8[8];
@@ -720,254 +718,316 @@ __global__ void __launch_bounds__(kTcThreads, 1) k_update_tc(const TcArgs<D> a) 
   tc::fence_after();
   const uint32_t tb = ms->tbase;
 
-  if (wid >= 8 && wid < kMmaWarp) {
+  if (wid >= 8 && wid < 8 + kProdWarps) {
     // ================================ producers ================================
-    // Thread pt owns entry slot pt of every entry tile.  While entry tile jt is built from
-    // the record staged in raw[jt&1][pt], the record of slot pt of tile jt+1 is fetched by
-    // asynchronous copies (cp.async, waited by the same thread: no cross-thread hand-off).
-    const int pt = tid - 256;  // 0..kProd-1
-    const int pw = wid - 8;
-    constexpr int R = C::R;
-    const int32_t* __restrict__ ent = a.ent + a.eoff[tile];
+    // Thread pt owns entry slot pt of every entry tile.  The unit of slot pt of tile t comes
+    // from the slot list (k_tc_expand).  (Walking the range list in the kernel instead was
+    // measured slower: its index work sits on the producers' critical path.)
+    const int pt = tid - 256;  // entry slot 0..127
+    const int pw = pt >> 5;
     const float Rq = ms->Rq, Rqi = ms->Rqi;
-    // records of slot pt of the next entry tile are copied while this one is built; the
-    // slot's unit index is loaded one more tile ahead so its latency is hidden as well
-    auto fetch = [&](int32_t c, int sb) {
-      if (c >= 0) {
-        float* dst = raw + ((size_t)sb * kTcEnt + pt) * R;
-        const float* src = a.c_rec + (int64_t)c * R;
-#pragma unroll
-        for (int k = 0; k < R / 4; ++k) cp_async16(dst + 4 * k, src + 4 * k);
+    const int nchunk = N2 / 16;
+    const int32_t* __restrict__ ent = a.ent + a.eoff[tile];
+    // copies of entry tile t into its stage (one cp.async group per tile, empty beyond T)
+    // Per entry tile t: the slot's unit (slot list, one tile ahead), then its record head (the
+    // 16-byte blocks of the block-major c_head: coalesced along a run of units) and digit row
+    // by cp.async straight into the stage, one tile ahead of the build.
+    constexpr int NH = R0 / 4;
+    // slot units are copied (cp.async, 4 bytes) three tiles ahead into a per-thread ring in
+    // shared memory, so the slot list's DRAM latency never sits in front of a fetch
+    int32_t* slotq = slots + pt;  // [4][kProd]: slot of tile t at slotq[(t & 3) * kProd]
+    auto slot_copy = [&](int t) {
+      if (t < T) {
+        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(tc::smem_addr(slotq + (t & 3) * kProd)),
+                     "l"(ent + (int64_t)t * kTcEnt + pt)
+                     : "memory");
       }
-      cp_async_commit();
     };
-    auto unit_of = [&](int jt) -> int32_t { return jt < T ? ent[(int64_t)jt * kTcEnt + pt] : -1; };
-    int32_t c_cur = unit_of(0), c_nxt = unit_of(1);
-    if (T > 0) fetch(c_cur, 0);
-    unsigned long long pc[4] = {0, 0, 0, 0};
-    for (int jt = 0; jt < T; ++jt) {
-      const int s = jt % NST, sb = jt & 1;
-      const int32_t c = c_cur;
-      long long t0 = clock64();
-      if (jt + 1 < T) {
-        fetch(c_nxt, sb ^ 1);
-        c_cur = c_nxt;
-        c_nxt = unit_of(jt + 2);
-      }
-      long long t1 = clock64();
-      if (jt >= NST) tc::bar_wait(&ms->stage_empty[s], ((jt / NST) - 1) & 1);  // overlaps the copies
-      long long t2 = clock64();
-      if (jt + 1 < T) cp_async_wait<1>();
-      else cp_async_wait<0>();
-      long long t3 = clock64();
-      pc[0] += t1 - t0;
-      pc[1] += t2 - t1;
-      pc[2] += t3 - t2;
-      pc[3] -= t3;
-      TcStage<D> st(ring, s);
-      const float* rb = raw + (size_t)sb * kTcEnt * R;
-      const float W = tc_build_entry<D>(a, ms, st, pt, c, rb + pt * R, Rq, Rqi);
-      float wm = W;
+    RingPos fp;  // stage of the tile being fetched
+    auto fetch = [&](int t) {  // copies for tile t (cp.async group, possibly empty); slot of t landed
+      if (t < T) {
+        const int32_t c = slotq[(t & 3) * kProd];
+        TCP_T(f0);
+        if (t >= NST) tc::bar_sleep(&ms->stage_empty[fp.i], fp.ph ^ 1u);
+        TCP_T(f1);
+        TCP_ADD(3, f1 - f0);
+        TcStage<D> st(ring, fp.i, SB, N2);
+        st.cell[pt] = c;
+        if (c >= 0) {
+          float* dst = st.rec + pt * C::R0S;
 #pragma unroll
-      for (int off = 16; off > 0; off >>= 1) wm = fmaxf(wm, __shfl_xor_sync(FULLMASK, wm, off));
-      if (lane == 0) st.wmax[pw] = wm;
+          for (int k = 0; k < NH; ++k) cp_async16(dst + 4 * k, a.c_head + ((int64_t)k * a.cap + c) * 4);
+          int8_t* b2 = st.b2 + pt * 16;
+          const int8_t* dg = a.c_dig + (int64_t)c * 16;
+#pragma unroll
+          for (int k = 0; k < C::DB / 16; ++k)
+            if (k < nchunk) cp_async16(b2 + k * (16 * kTcEnt), dg + (int64_t)k * a.cap * 16);
+        }
+        fp.adv(NST);
+      }
+    };
+    // prologue: slots of tiles 0..2, then tile 0's copies (group 0 also carries slot 3)
+    slot_copy(0);
+    slot_copy(1);
+    slot_copy(2);
+    cp_async_commit();
+    cp_async_wait<0>();
+    fetch(0);
+    slot_copy(3);
+    cp_async_commit();
+    RingPos bp;  // stage of the tile being built
+    for (int jt = 0; jt < T; ++jt) {
+      TCP_T(p0);
+      fetch(jt + 1);                // next tile's copies in flight during this build
+      slot_copy(jt + 4);
+      cp_async_commit();
+      TCP_T(p1);
+      TCP_ADD(0, p1 - p0);
+      cp_async_wait<1>();           // this tile's record heads and digit rows (and slot jt+3) landed
+      TCP_T(p2);
+      TCP_ADD(1, p2 - p1);
+      TcStage<D> st(ring, bp.i, SB, N2);
+      const float W = tc_build_entry<D>(a, ms, st, pt, st.cell[pt], st.rec + pt * C::R0S, Rq, Rqi);
+      // chunk maximum of the band widths (W >= 0: its bits order as unsigned integers)
+      const uint32_t wm = __reduce_max_sync(FULLMASK, __float_as_uint(W));
+      if (lane == 0) st.wmax[pw] = __uint_as_float(wm);
       tc::fence_proxy_async();
-      tc::bar_arrive(&ms->stage_full[s]);
-      pc[3] += clock64();
-    }
-    if (a.prof && tid == 256) {
-      for (int k = 0; k < 4; ++k) atomicAdd(&a.prof[k], pc[k]);
-      atomicAdd(&a.prof[4], (unsigned long long)T);
+      tc::bar_arrive(&ms->stage_full[bp.i]);
+      bp.adv(NST);
+      TCP_T(p3);
+      TCP_ADD(2, p3 - p2);
     }
   }
 
-  if (wid == kMmaWarp) {
-    // ================================ MMA issue ================================
-    // One thread issues, in order (the tensor pipe executes them in order):
-    //   GEMM1(jt)        S[jt % NS] = Q . B1(jt)^T      once stage jt is built
-    //   GEMM2(jt-NS+1)   O[g] (+)= P . B2^T             once its classifier group wrote P
-    // so GEMM1 runs NS-1 tiles ahead of the classifiers and GEMM1(jt) follows GEMM2(jt-NS),
-    // the last reader of its S buffer.  Blocking waits (the warp is suspended, it does not
-    // take issue slots from the classifier / producer warps of its sub-partition).
-    if (lane == 0) {
-      constexpr uint32_t id1 = tc::idesc_tf32(128, kTcEnt, false);
-      constexpr uint32_t id2 = tc::idesc_tf32(128, N2, false);
-      constexpr int NS = C::kNS;
-      const uint32_t ring_s = tc::smem_addr(ring);
-      const int T0 = (T + 1) / 2, T1 = T / 2;  // entry tiles of group 0 / 1
-      for (int jt = 0; jt < T + NS - 1; ++jt) {
-        if (jt < T) {
-          const int s = jt % NST, sb = jt % NS;
-          tc::bar_wait(&ms->stage_full[s], (jt / NST) & 1);
-          tc::fence_after();
-          const uint32_t b1 = ring_s + s * C::kStageBytes;
+  if (wid == kMma1Warp && lane == 0) {
+    // ================================ GEMM1 issue ================================
+    // S[jt % NS] = Q . B1(jt)^T once stage jt is built and GEMM2(jt - NS) released the buffer.
+    constexpr uint32_t id1 = tc::idesc_tf32(128, kTcEnt, false);
+    const uint32_t ring_s = tc::smem_addr(ring);
+    RingPos sp, bq;
+    for (int jt = 0; jt < T; ++jt) {
+      const int s = sp.i, b = bq.i;
+      TCP_T(m0);
+      tc::bar_sleep(&ms->stage_full[s], sp.ph);
+      TCP_T(m1);
+      if (jt >= NS) tc::bar_sleep(&ms->s_free[b], bq.ph ^ 1u);
+      TCP_T(m2);
+      TCP_ADD(0, m1 - m0);
+      TCP_ADD(1, m2 - m1);
+      tc::fence_after();
+      const uint32_t b1 = ring_s + s * SB;
 #pragma unroll
-          for (int k = 0; k < K1 / 8; ++k)
-            tc::mma_ts(tb + C::kColS + kTcEnt * sb, tb + C::kColQ + 8 * k, tc::sdesc(b1 + k * 256, 128, C::SBO1), id1,
-                       k > 0);
-          tc::mma_commit(&ms->s_full[sb]);
-        }
-        const int jj = jt - (NS - 1);
-        if (jj >= 0 && jj < T) {
-          const int s = jj % NST, sb = jj % NS, g = jj & 1, kk = jj >> 1;
-          tc::bar_wait(&ms->p_full[sb], (jj / NS) & 1);  // per S buffer: never two phases ahead
-          tc::fence_after();
-          const uint32_t b2 = ring_s + s * C::kStageBytes + C::kB1Bytes;
-          const uint32_t acc0 = (kk % kDrain) != 0;
-#pragma unroll
-          for (int k = 0; k < kTcEnt / 8; ++k)
-            tc::mma_ts(tb + C::kColO + N2 * g, tb + C::kColS + kTcEnt * sb + 8 * k,
-                       tc::sdesc(b2 + k * 2 * C::LBO2, C::LBO2, C::SBO2), id2, (k > 0) || acc0);
-          tc::mma_commit(&ms->stage_empty[s]);
-          const int Tg = g ? T1 : T0;
-          if ((kk % kDrain) == kDrain - 1 || kk == Tg - 1) tc::mma_commit(&ms->o_full[g]);
-        }
-      }
+      for (int k = 0; k < K1 / 8; ++k)
+        tc::mma_ts(tb + kColS + kTcEnt * b, tb + 8 * k, tc::sdesc(b1 + k * 256, 128, C::SBO1), id1, k > 0);
+      tc::mma_commit(&ms->s_full[b]);
+      sp.adv(NST);
+      bq.adv(NS);
     }
-    __syncwarp();
+  }
+  if (wid == kMma2Warp && lane == 0) {
+    // ================================ GEMM2 issue ================================
+    // O += P . B2(jt)^T (int8 x int8 -> int32, exact) once a classifier group wrote P(jt)
+    // into the first 32 columns of S[jt % NS]; releases the stage and the S buffer.
+    const uint32_t id2 = tc::idesc_s8(128, N2, true);
+    const uint32_t ring_s = tc::smem_addr(ring);
+    RingPos sp, bq;
+    for (int jt = 0; jt < T; ++jt) {
+      const int s = sp.i, b = bq.i;
+      TCP_T(m0);
+      tc::bar_sleep(&ms->p_full[b], bq.ph);
+      TCP_T(m1);
+      TCP_ADD(0, m1 - m0);
+      tc::fence_after();
+      const uint32_t b2 = ring_s + s * SB + C::kB1Bytes;
+#pragma unroll
+      for (int k = 0; k < kTcEnt / 32; ++k)
+        tc::mma_ts_s8(tb + kColO, tb + kColS + kTcEnt * b + 8 * k, tc::sdesc(b2 + k * 512, 128, 16 * kTcEnt), id2,
+                      (jt > 0) || (k > 0));
+      tc::mma_commit(&ms->stage_empty[s]);
+      tc::mma_commit(&ms->s_free[b]);
+      sp.adv(NST);
+      bq.adv(NS);
+    }
+    tc::mma_commit(&ms->o_done);
   }
 
   if (is_cls) {
     // ================================ classifiers ================================
     const uint32_t lane_off = (uint32_t)(32 * (wid & 3)) << 16;
     const int Tg = grp ? T / 2 : (T + 1) / 2;
-    unsigned long long* racc = rare + grp * (NV + 1) * kTcTile;  // this group's sums (rows are exclusive)
-    int dc = 0;  // drains done
-    unsigned long long cw[3] = {0, 0, 0};
-    // O (fp32, <= kDrain entry tiles) -> the row's exact fixed-point sums in shared memory
-    // (integer atomics: both groups add to the same rows, order-independent)
-    auto drain = [&]() {
-      tc::bar_wait(&ms->o_full[grp], dc & 1);
-      ++dc;
+    const float lim_in = a.e2f * (1.f - a.rel), lim_out = a.e2f * (1.f + a.rel);
+    RingPos sp, bq;  // stage / S buffer of tile jt = 2 kk + grp
+    if (grp) {
+      sp.adv(NST);
+      bq.adv(NS);
+    }
+    for (int kk = 0; kk < Tg; ++kk) {
+      const int s = sp.i, b = bq.i;
+      TcStage<D> st(ring, s, SB, N2);
+      TCP_T(c0);
+      tc::bar_sleep(&ms->s_full[b], bq.ph);
+      TCP_T(c1);
+      TCP_ADD(0, c1 - c0);
       tc::fence_after();
-      double hi[NV];
+      const uint32_t sb = tb + lane_off + kColS + kTcEnt * b;
+#pragma unroll 1
+      for (int cp = 0; cp < kTcEnt / 64; ++cp) {
+        uint32_t v[2][32];
+        tc::ld32(sb + 64 * cp, v[0]);
+        tc::ld32(sb + 64 * cp + 32, v[1]);
+        TCP_T(l0);
+        tc::wait_ld();
+        TCP_T(l1);
+        TCP_ADD(1, l1 - l0);
+        uint32_t pw[16];
 #pragma unroll
-      for (int c = 0; c < N2 / 16; ++c) {
+        for (int h = 0; h < 2; ++h) {
+          const int c = 2 * cp + h;
+          const uint32_t wm = __float_as_uint(st.wmax[c]);
+          uint32_t mn = 0xFFFFFFFFu;
+#pragma unroll
+          for (int jx = 0; jx < 32; ++jx) {
+            v[h][jx] = __float_as_uint(__uint_as_float(v[h][jx]) + pp);  // |p - c_e|^2 - limF_e
+            mn = min(mn, v[h][jx]);  // unsigned: negative values (inside) compare large
+          }
+#pragma unroll
+          for (int w = 0; w < 8; ++w)
+            pw[8 * h + w] = sign_bytes4(v[h][4 * w], v[h][4 * w + 1], v[h][4 * w + 2], v[h][4 * w + 3]);
+          TCP_T(b0);
+          if (mn < wm) {  // some pair of this chunk may lie in a band (0 <= f <= max W): exact decisions
+            uint32_t bm = 0u;
+#pragma unroll
+            for (int jx = 0; jx < 32; ++jx) bm |= (v[h][jx] < wm) ? (1u << jx) : 0u;
+            uint32_t fm = 0u;  // band pairs decided inside (single points)
+            while (bm) {
+              const int jx = __ffs(bm) - 1;
+              bm &= bm - 1u;
+              const int e = 32 * c + jx;
+              if (st.cnt(e) == 1) {
+                float qc[D];
+#pragma unroll
+                for (int i = 0; i < D; ++i) qc[i] = st.pt(e, i);
+                // a single point: fp32 distance from the exact coordinates decides unless it lies
+                // within the (4D+16)u margin of eps^2 (as k_update); there Def. of N_eps (L66)
+                // exactly as the oracle: fp64, dimension order
+                float d2 = 0.f;
+#pragma unroll
+                for (int i = 0; i < D; ++i) {
+                  const float u = qc[i] - pe[i];
+                  d2 = fmaf(u, u, d2);
+                }
+                bool in = d2 <= lim_in;
+                if (!in && d2 <= lim_out) {
+                  double s2 = 0.0;
+#pragma unroll
+                  for (int i = 0; i < D; ++i) {
+                    const double t = __dsub_rn((double)qc[i], (double)pe[i]);
+                    s2 = __dadd_rn(s2, __dmul_rn(t, t));
+                  }
+                  in = s2 <= a.e2d;
+                }
+                if (in) fm |= 1u << jx;
+              } else {
+                tc_rare<D>(a, pe, e, st, rare, row);
+              }
+            }
+#pragma unroll
+            for (int w = 0; w < 8; ++w) {
+              const uint32_t f4 = (fm >> (4 * w)) & 0xFu;
+              pw[8 * h + w] |= (f4 & 1u ? 0xFFu : 0u) | (f4 & 2u ? 0xFF00u : 0u) | (f4 & 4u ? 0xFF0000u : 0u) |
+                               (f4 & 8u ? 0xFF000000u : 0u);
+            }
+          }
+          TCP_T(b1);
+          TCP_ADD(2, b1 - b0);
+        }
+        tc::st16(sb + 16 * cp, pw);  // P (int8, -1 = inside) over S columns already read
+      }
+      TCP_T(w0);
+      tc::wait_st();
+      TCP_T(w1);
+      TCP_ADD(3, w1 - w0);
+      tc::fence_before();
+      tc::bar_arrive(&ms->p_full[b]);
+      sp.adv(NST);
+      sp.adv(NST);
+      bq.adv(NS);
+      bq.adv(NS);
+    }
+  }
+#ifdef EGG_TC_PROF
+  // one reporting thread per role: classifiers 0 / 128, producer 256, GEMM1 / GEMM2 issuers
+  {
+    int slot = -1;
+    if (tid == 0 || tid == 128) slot = 0;
+    else if (tid == 256) slot = 4;
+    else if (wid == kMma1Warp && lane == 0) slot = 8;
+    else if (wid == kMma2Warp && lane == 0) slot = 12;
+    if (slot >= 0 && a.prof)
+      for (int k = 0; k < (slot == 12 ? 1 : 4); ++k) atomicAdd(&a.prof[slot + k], prof_acc[k]);
+    if (tid == 0 && a.prof) atomicAdd(&a.prof[15], (unsigned long long)T);
+  }
+#endif
+
+  // ---- epilogue (group 0 rows): Eq.5 in fp64 from the exact integer sums ----------------
+  __syncthreads();  // every role done issuing / classifying
+  if (is_cls && grp == 0) {
+    tc::bar_sleep(&ms->o_done, 0);
+    tc::fence_after();
+    if (T > 0) {
+      // O[k*NV + jv] = -(sum over inside entries of digit k of value jv): fold into the row's
+      // fixed-point sums (mod 2^64 arithmetic: exact since every total fits in int64)
+      const uint32_t lane_off = (uint32_t)(32 * (wid & 3)) << 16;
+      const int used = a.ndig * NV;
+      for (int c16 = 0; c16 < N2 / 16; ++c16) {
         uint32_t v[16];
-        tc::ld16(tb + lane_off + C::kColO + N2 * grp + 16 * c, v);
+        tc::ld16(tb + lane_off + kColO + 16 * c16, v);
         tc::wait_ld();
 #pragma unroll
         for (int jx = 0; jx < 16; ++jx) {
-          const int col = 16 * c + jx;
-          const float f = __uint_as_float(v[jx]);
-          if (col < NV) {
-            hi[col] = (double)f;
-          } else if (col < 2 * NV) {
-            const int i = col - NV;
-            if (i < 2 * D) {
-              const double x = hi[i] + (double)f;
-              racc[i * kTcTile + row] += (unsigned long long)llrint(x * kFix);
-            } else {  // count: exact integers in both halves
-              const long long nc = llrint(hi[i]) + llrint((double)f);
-              racc[NV * kTcTile + row] += (unsigned long long)nc;
-            }
+          const int col = 16 * c16 + jx;
+          if (col < used) {
+            const int k = col / NV, jv = col - k * NV;
+            const unsigned long long t = (unsigned long long)(long long)(int32_t)v[jx];
+            const int sh = jv < 2 * D ? 8 * k + (32 - kDigF) : 8 * k;
+            rare[jv * kTcTile + row] -= t << sh;
           }
         }
       }
-    };
-    for (int kk = 0; kk < Tg; ++kk) {
-      const int jt = 2 * kk + grp;
-      const int s = jt % NST, sb = jt % C::kNS;
-      TcStage<D> st(ring, s);
-      long long c0 = clock64();
-      tc::bar_wait(&ms->s_full[sb], (jt / C::kNS) & 1);
-      tc::fence_after();
-      long long c1 = clock64();
-      cw[0] += c1 - c0;
-#pragma unroll 1
-      for (int c = 0; c < kTcEnt / 32; ++c) {
-        const uint32_t taddr = tb + lane_off + C::kColS + kTcEnt * sb + 32 * c;
-        uint32_t v[32];
-        tc::ld32(taddr, v);
-        tc::wait_ld();
-        const uint32_t wm = __float_as_uint(st.wmax[c]);
-        uint32_t mn = 0xFFFFFFFFu;
+    }
+    if (valid) {
+      auto fx = [&](int k) { return (long long)rare[k * kTcTile + row]; };
+      const int64_t Ni = fx(2 * D) + (int64_t)a.full_N[j];
+      const double inv = 1.0 / (double)Ni;
 #pragma unroll
-        for (int jx = 0; jx < 32; ++jx) {
-          const float f = __uint_as_float(v[jx]) + pp;  // |p - c_e|^2 - limF_e
-          v[jx] = __float_as_uint(f);
-          mn = __viaddmin_u32(v[jx], 0xFFFFFFFFu, mn);  // min over f > 0 of bits(f) - 1
-        }
-        if (mn < wm) {  // some pair of this chunk may lie in a band: exact decisions
-          // candidates 0 < f <= max band of the chunk (bit trick as for mn); a candidate
-          // outside its own entry's band is still decided exactly below (same answer)
-          uint32_t bm = 0u;
-#pragma unroll
-          for (int jx = 0; jx < 32; ++jx) bm |= (v[jx] - 1u < wm) ? (1u << jx) : 0u;
-          uint32_t fm = 0u;  // band pairs decided inside (single points)
-          while (bm) {
-            const int jx = __ffs(bm) - 1;
-            bm &= bm - 1u;
-            const int e = 32 * c + jx;
-            if (st.cnt[e] == 1) {  // Def. of N_eps (L66) exactly as the oracle: fp64, dimension order
-              double s2 = 0.0;
-#pragma unroll
-              for (int i = 0; i < D; ++i) {
-                const double t = __dsub_rn((double)a.xs[(int64_t)i * a.n + st.start[e]], (double)pe[i]);
-                s2 = __dadd_rn(s2, __dmul_rn(t, t));
-              }
-              if (s2 <= a.e2d) fm |= 1u << jx;
-            } else {
-              tc_rare<D>(a, pe, e, st, racc, row);
-            }
-          }
-#pragma unroll
-          for (int jx = 0; jx < 32; ++jx)
-            v[jx] = (__uint_as_float(v[jx]) <= 0.f || ((fm >> jx) & 1u)) ? 0x3F800000u : 0u;
-        } else {
-#pragma unroll
-          for (int jx = 0; jx < 32; ++jx) v[jx] = __uint_as_float(v[jx]) <= 0.f ? 0x3F800000u : 0u;
-        }
-        tc::st32(taddr, v);
+      for (int i = 0; i < D; ++i) {
+        const double S = (double)fx(i) * kInvFix + a.full_S[(int64_t)i * a.n + j];
+        const double Cc = (double)fx(D + i) * kInvFix + a.full_S[(int64_t)(D + i) * a.n + j];
+        double sx, cx;
+        const double x = (double)pe[i];
+        sincos(x, &sx, &cx);
+        const double xn = x + (cx * S - sx * Cc) * inv;  // Eq.5
+        a.xs_next[(int64_t)i * a.n + j] = (float)xn;
       }
-      tc::wait_st();
-      long long c2 = clock64();
-      cw[1] += c2 - c1;
-      if (kk >= 1 && ((kk - 1) % kDrain) == kDrain - 1) drain();
-      cw[2] += clock64() - c2;
-      tc::fence_before();
-      tc::bar_arrive(&ms->p_full[sb]);
+      const bool f1 = Ni == (int64_t)a.g_cnt[a.g_of[j]];  // Alg 3 l.14-15 (L248)
+      if (!f1) atomicAnd(&a.flags[0], 0);
+      if (a.nbr) a.nbr[j] = (int32_t)Ni;
     }
-    if (Tg > 0) drain();
-    if (a.prof && (tid == 0 || tid == 128)) {
-      for (int k = 0; k < 3; ++k) atomicAdd(&a.prof[5 + k], cw[k]);
-    }
-  }
-
-  // ---- epilogue (group 0 rows): Eq.5 in fp64 from the exact fixed-point sums -------------
-  __syncthreads();  // all MMAs drained
-  if (is_cls && grp == 0 && valid) {
-    const unsigned long long* r0 = rare;
-    const unsigned long long* r1 = rare + (NV + 1) * kTcTile;
-    auto fx = [&](int k) { return (long long)(r0[k * kTcTile + row] + r1[k * kTcTile + row]); };
-    const int64_t Nt = fx(NV);  // tensor-core count
-    const int64_t Ni = Nt + fx(2 * D) + (int64_t)a.full_N[j];
-    const double inv = 1.0 / (double)Ni;
-#pragma unroll
-    for (int i = 0; i < D; ++i) {
-      const double S = (double)Nt * (double)ms->s0[i] + (double)fx(i) * kInvFix + a.full_S[(int64_t)i * a.n + j];
-      const double Cc = (double)Nt * (double)ms->c0[i] + (double)fx(D + i) * kInvFix + a.full_S[(int64_t)(D + i) * a.n + j];
-      double sx, cx;
-      const double x = (double)pe[i];
-      sincos(x, &sx, &cx);
-      const double xn = x + (cx * S - sx * Cc) * inv;  // Eq.5
-      a.xs_next[(int64_t)i * a.n + j] = fminf(fmaxf((float)xn, 0.f), 1.f);
-    }
-    const bool f1 = Ni == (int64_t)a.g_cnt[a.g_of[j]];  // Alg 3 l.14-15 (L248)
-    if (!f1) atomicAnd(&a.flags[0], 0);
-    if (a.nbr) a.nbr[j] = (int32_t)Ni;
   }
   tc::fence_before();
   __syncthreads();
-  if (wid == kMmaWarp) {
+  if (wid == kMma1Warp) {
     tc::fence_after();
     tc::tmem_dealloc<512>(tb);
   }
 }
-
 // ----------------------------------------------------------------------------------------
 // host side
 // ----------------------------------------------------------------------------------------
+template <int D>
+int run_planned_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr, int64_t owned);
+inline bool tc_choose(const long long* g);
+
 template <int D>
 int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   if constexpr (D > kTcMaxD) {
@@ -978,7 +1038,13 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     const int64_t owned =
         ntot > ws.own_offset ? (ntot - ws.own_offset + ws.own_stride - 1) / ws.own_stride : 0;
     ws.tc_used = 1;
-    if (owned == 0) return EGGSYNC_OK;
+    if (ws.tc_mode == 2) return run_planned_tc<D>(ws, lo, hi, nbr, owned);
+    if (owned == 0) {
+      for (auto& v : ws.tc_local) v = 0;
+      ws.tc_local[5] = 1;
+      ws.tc_pad = 0;
+      return EGGSYNC_OK;
+    }
     PlanArgs<D> p;
     p.xs = ws.xs[ws.xcur];
     p.t_meta = ws.t_meta;
@@ -1011,44 +1077,62 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     const size_t psmem = (size_t)kPlanWarps * p.stack_len * 8 * sizeof(int);
     const unsigned pgrid = (unsigned)((owned + kPlanWarps - 1) / kPlanWarps);
     EGG_CUDA(cudaFuncSetAttribute(k_tc_plan<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)psmem));
-    p.t_epad = ws.tc_epad;
     p.t_pv = ws.tc_pv;
     // the range buffer keeps its size across updates (process cache); a first guess of
     // 16 chunks per tile, grown and re-planned when the plan reports more
     EGG_TRY(tc_ranges_reserve(ws, (size_t)owned * 16 * kRangeChunk));
+    p.t_epad = ws.tc_epad;
     size_t tmp = 0;
     EGG_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tmp, ws.tc_epad, ws.tc_eoff, (int)owned + 1, ws.stream));
     if (tmp > ws.cub_bytes) {
       set_error("cub scratch too small for the tensor-core plan scan");
       return EGGSYNC_ECUDA;
     }
-    int32_t hc[7] = {0, 0, 0, 0, 0, 0, 0};  // ctr[0..5], padded entries
+    int32_t hc[10] = {0, 0, 0, 0, 0, 0, 0, 0, 0, 0};  // ctr[0..7] (padded entries at 6..7), largest cell count
     for (int attempt = 0; attempt < 2; ++attempt) {
       p.ranges = ws.tc_ranges;
       p.rcap = (int64_t)ws.tc_rcap;
-      EGG_CUDA(cudaMemsetAsync(ws.tc_ctr, 0, 6 * sizeof(int32_t), ws.stream));
+      EGG_CUDA(cudaMemsetAsync(ws.tc_ctr, 0, 8 * sizeof(int32_t), ws.stream));
       EGG_CUDA(cudaMemsetAsync(ws.tc_epad + owned, 0, sizeof(int32_t), ws.stream));
       k_tc_plan<D><<<pgrid, kPlanWarps * 32, psmem, ws.stream>>>(p);
       EGG_CUDA(cudaGetLastError());
       EGG_CUDA(cub::DeviceScan::ExclusiveSum(ws.cub_tmp, tmp, ws.tc_epad, ws.tc_eoff, (int)owned + 1, ws.stream));
-      EGG_CUDA(cudaMemcpyAsync(hc, ws.tc_ctr, 6 * sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
-      EGG_CUDA(cudaMemcpyAsync(hc + 6, ws.tc_eoff + owned, sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
+      ws.launches += 2;
+      EGG_CUDA(cudaMemcpyAsync(hc, ws.tc_ctr, 8 * sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
+      EGG_CUDA(cudaMemcpyAsync(hc + 8, ws.flags + 5, sizeof(int32_t), cudaMemcpyDeviceToHost, ws.stream));
       EGG_CUDA(cudaStreamSynchronize(ws.stream));
-      ws.launches += 3;  // plan + scan (2)
+      ws.launches += 1;
       if (hc[1] || (size_t)(uint32_t)hc[0] <= ws.tc_rcap) break;
       EGG_TRY(tc_ranges_reserve(ws, (size_t)(uint32_t)hc[0]));
     }
-    if (hc[1] || (size_t)(uint32_t)hc[0] > ws.tc_rcap) {  // a tile with > kChunkMax chunks: SIMT kernel
-      ws.tc_used = 0;
-      return run_update_simt<D>(ws, lo, hi, nbr);
-    }
-    unsigned long long ent_u = 0, pts_u = 0;
+    unsigned long long ent_u = 0, pts_u = 0, pad_u = 0;
     memcpy(&ent_u, hc + 2, sizeof(ent_u));
     memcpy(&pts_u, hc + 4, sizeof(pts_u));
-    const double occ = ent_u ? (double)pts_u / (double)ent_u : 1.0;
+    memcpy(&pad_u, hc + 6, sizeof(pad_u));
+    // a tile with > kChunkMax chunks, or a range buffer still too small: the plan is unusable
+    const bool overflow = hc[1] || (size_t)(uint32_t)hc[0] > ws.tc_rcap;
+    ws.tc_local[0] = (long long)ent_u;
+    ws.tc_local[1] = (long long)pts_u;
+    ws.tc_local[2] = owned;
+    ws.tc_local[3] = overflow ? 1 : 0;
+    ws.tc_local[4] = hc[8];
+    ws.tc_local[5] = 1;
+    ws.tc_pad = (long long)pad_u;
     if (getenv("EGGSYNC_TC_DEBUG"))
-      fprintf(stderr, "[tc-plan] entries=%llu points_in_entries=%llu ratio=%.3f slots=%d overflow=%d padded=%d rcap=%zu tiles=%lld\n",
-              ent_u, pts_u, occ, hc[0], hc[1], hc[6], ws.tc_rcap, (long long)owned);
+      fprintf(stderr, "[tc-plan] entries=%llu points_in_entries=%llu slots=%d overflow=%d padded=%d rcap=%zu tiles=%lld\n",
+              ent_u, pts_u, hc[0], hc[1], (int)pad_u, ws.tc_rcap, (long long)owned);
+    if (ws.tc_mode == 1) return EGGSYNC_OK;  // plan only: the ranks choose the kernel together
+    return run_planned_tc<D>(ws, lo, hi, nbr, owned);
+  }
+}
+
+// The kernel choice from plan statistics (summed over all ranks in a multi-rank update, so that
+// every rank and a single GPU choose alike), then the tensor-core update of the local plan.
+inline bool tc_choose(const long long* g) {
+  if (!g[5] || g[3]) return false;  // tensor cores not enabled / a rank's plan overflowed
+  const unsigned long long ent = (unsigned long long)g[0], pts = (unsigned long long)g[1],
+                           tiles = (unsigned long long)g[2];
+  const double occ = ent ? (double)pts / (double)ent : 1.0;
     // Entries holding a few points each on average (partly collapsed clusters) put many
     // multi-point cells in the classifiers' exact band, where one lane scans a cell's points
     // alone; the warp-cooperative SIMT kernel is faster there (measured: C4-d10 iterations
@@ -1058,12 +1142,25 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     // (e.g. C5 iteration 1: 2.5e10 entries, 3e12 pairs) the SIMT kernel runs instead; so it
     // does when the tiles average less than one entry tile (a CTA per nearly empty tile:
     // C5 iteration 3, 13 entries per tile, 14 ms vs 2 ms).
-    if ((occ > 1.1 && occ < 50.0) || ent_u + (unsigned long long)owned * kTcEnt > (1ull << 30) ||
-        ent_u < (unsigned long long)owned * kTcEnt) {
+  return !((occ > 1.1 && occ < 50.0) || ent + tiles * kTcEnt > (1ull << 30) || ent < tiles * kTcEnt);
+}
+
+template <int D>
+int run_planned_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr, int64_t owned) {
+  if constexpr (D > kTcMaxD) {
+    return EGGSYNC_EINVAL;
+  } else {
+    using C = TcCfg<D>;
+    if (!tc_choose(ws.tc_mode == 2 ? ws.tc_global : ws.tc_local)) {
       ws.tc_used = 0;
       return run_update_simt<D>(ws, lo, hi, nbr);
     }
-    EGG_TRY(tc_ent_reserve(ws, (size_t)(uint32_t)hc[6] + 1));
+    ws.tc_used = 1;
+    if (owned == 0) return EGGSYNC_OK;
+    const unsigned long long ent_u = (unsigned long long)ws.tc_local[0], pad_u = (unsigned long long)ws.tc_pad;
+    int32_t hc[10];
+    hc[8] = (int32_t)(ws.tc_mode == 2 ? ws.tc_global[4] : ws.tc_local[4]);
+    EGG_TRY(tc_ent_reserve(ws, (size_t)pad_u + 1));
     k_tc_expand<0><<<(unsigned)((owned + 3) / 4), 128, 0, ws.stream>>>(ws.tc_ranges, ws.tc_chunks, ws.tc_nr, ws.tc_ne,
                                                                     ws.tc_eoff, ws.tc_ent, (int32_t)owned);
     EGG_CUDA(cudaGetLastError());
@@ -1082,6 +1179,22 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
       ws.launches += 4;
     }
 
+    // GEMM2 layout: digits per summary value from the largest cell count (balanced base-256
+    // digits of |v| <= count * 2^kDigF hold 0.498 * 2^(8k)), N = digits * (2D+1) -> x16
+    const long long maxc = hc[8] > 1 ? hc[8] : 1;
+    int ndig = 3;
+    while (ndig < kDigMax && (double)maxc * (double)(1 << kDigF) + 1.0 > 0.498 * std::ldexp(1.0, 8 * ndig)) ++ndig;
+    const int n2 = (ndig * C::NV + 15) / 16 * 16;
+    const int ns = (C::K1 + 3 * kTcEnt + n2 <= 512) ? 3 : 2;  // S buffers that fit TMEM next to Q and O
+    const int sbytes = C::stage_bytes(n2);
+    int nst = (C::kBudget - C::kFixedBytes) / sbytes;
+    nst = nst > kTcMaxStages ? kTcMaxStages : nst;
+    if (nst < 2 || C::K1 + 2 * kTcEnt + n2 > 512) {  // cannot happen for D <= kTcMaxD
+      ws.tc_used = 0;
+      return run_update_simt<D>(ws, lo, hi, nbr);
+    }
+    const size_t smem = (size_t)nst * sbytes + C::kFixedBytes;
+
     TcArgs<D> a;
     a.xs = ws.xs[ws.xcur];
     a.xs_next = ws.xs[ws.xcur ^ 1];
@@ -1090,6 +1203,9 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     a.g_of = ws.g_of;
     a.g_cnt = ws.g_cnt;
     a.c_rec = ws.c_rec;
+    a.c_dig = ws.c_dig;
+    a.c_head = ws.c_head;
+    a.cell_of = ws.cell_of;
     a.c_lo = ws.c_lo;
     a.c_hi = ws.c_hi;
     a.ent = ws.tc_ent;
@@ -1105,46 +1221,57 @@ int run_update_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
     a.ntiles = (int32_t)owned;
     a.stride = ws.own_stride;
     a.offset = ws.own_offset;
+    a.ndig = ndig;
+    a.n2 = n2;
+    a.nst = nst;
+    a.ns = ns;
+    a.stage_bytes = sbytes;
     a.e = ws.k.ef;
     a.e2f = ws.k.e2f;
     a.rel = ws.k.rel;
     a.e2d = ws.k.e2;
     a.flags = ws.flags;
     a.nbr = nbr;
-    a.prof = nullptr;
-    static unsigned long long* prof = nullptr;
-    if (getenv("EGGSYNC_TC_PROF")) {
-      if (!prof) EGG_CUDA(cudaMalloc((void**)&prof, 16 * sizeof(unsigned long long)));
-      EGG_CUDA(cudaMemsetAsync(prof, 0, 16 * sizeof(unsigned long long), ws.stream));
-      a.prof = prof;
-    }
-    EGG_CUDA(cudaFuncSetAttribute(k_update_tc<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)C::kSmem));
+    EGG_CUDA(cudaFuncSetAttribute(k_update_tc<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
     if (ws.tc_timing) {
       EGG_TRY(ws.tc_flush());
-      const long long pairs = (long long)ent_u * kTcTile, padded = (long long)(uint32_t)hc[6] * kTcTile;
+      const long long pairs = (long long)ent_u * kTcTile, padded = (long long)pad_u * kTcTile;
       ws.tc_acc[0] += 1;
       ws.tc_acc[1] += pairs;
       ws.tc_acc[2] += padded;
-      // algorithmic tensor-core FLOPs: GEMM1 over the 3D+2 operand columns, GEMM2 over the
-      // 2(2D+1) value columns (hi/lo split), per (point, entry) pair
-      ws.tc_pend_alg = 2LL * pairs * ((3 * D + 2) + 2 * (2 * D + 1));
+      // tensor-core operations per (point, entry) pair as executed: GEMM1 over the 3D+2 tf32
+      // operand columns (hi/lo splits), GEMM2 over the digits x (2D+1) int8 value columns
+      ws.tc_pend_alg = 2LL * pairs * ((3 * D + 2) + ndig * C::NV);
       ws.tc_acc[3] += ws.tc_pend_alg;
       EGG_CUDA(cudaEventRecord(ws.tc_ev[0], ws.stream));
     }
-    k_update_tc<D><<<(unsigned)owned, kTcThreads, C::kSmem, ws.stream>>>(a);
+    if (getenv("EGGSYNC_TC_DEBUG"))
+      fprintf(stderr, "[tc-cfg] ndig=%d n2=%d stages=%d sbuf=%d stage_bytes=%d smem=%zu max_cell=%d\n", ndig, n2, nst,
+              ns, sbytes, smem, hc[8]);
+    a.prof = nullptr;
+#ifdef EGG_TC_PROF
+    static unsigned long long* prof = nullptr;
+    if (!prof) EGG_CUDA(cudaMalloc((void**)&prof, 16 * sizeof(unsigned long long)));
+    EGG_CUDA(cudaMemsetAsync(prof, 0, 16 * sizeof(unsigned long long), ws.stream));
+    a.prof = prof;
+#endif
+    k_update_tc<D><<<(unsigned)owned, kTcThreads, smem, ws.stream>>>(a);
     EGG_CUDA(cudaGetLastError());
-    if (ws.tc_timing) {
-      EGG_CUDA(cudaEventRecord(ws.tc_ev[1], ws.stream));
-      ws.tc_pending = true;
-    }
-    if (a.prof) {
+#ifdef EGG_TC_PROF
+    {
       unsigned long long h[16];
       EGG_CUDA(cudaMemcpyAsync(h, prof, sizeof(h), cudaMemcpyDeviceToHost, ws.stream));
       EGG_CUDA(cudaStreamSynchronize(ws.stream));
-      const double t = (double)(h[4] ? h[4] : 1);
-      fprintf(stderr, "[tc-prof] per entry tile (clk): producer fetch %.0f wait_empty %.0f wait_records %.0f build %.0f | "
-              "classifier wait_S %.0f classify %.0f drain %.0f\n", h[0] / t, h[1] / t, h[2] / t, h[3] / t,
-              2 * h[5] / t, 2 * h[6] / t, 2 * h[7] / t);
+      const double t = (double)(h[15] ? h[15] : 1);
+      fprintf(stderr, "[tc-prof] clk per entry tile: producer fetch %.0f (stage wait %.0f) wait_copies %.0f build %.0f | "
+              "classifier (per own tile) wait_S %.0f ld %.0f band %.0f wait_st %.0f | GEMM1 wait_full %.0f wait_free %.0f | "
+              "GEMM2 wait_P %.0f\n", h[4] / t, h[7] / t, h[5] / t, h[6] / t, h[0] / t, h[1] / t, h[2] / t, h[3] / t, h[8] / t,
+              h[9] / t, h[12] / t);
+    }
+#endif
+    if (ws.tc_timing) {
+      EGG_CUDA(cudaEventRecord(ws.tc_ev[1], ws.stream));
+      ws.tc_pending = true;
     }
     if (getenv("EGGSYNC_TC_DEBUG")) {
       std::vector<int32_t> h((size_t)owned);
@@ -1180,8 +1307,12 @@ inline bool tc_enabled(const Workspace& ws, int d) {
 template <int D>
 int run_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   ws.tc_used = 0;
+  if (tc_enabled(ws, D) && hi > lo) return run_update_tc<D>(ws, lo, hi, nbr);
+  if (ws.tc_mode == 1) {  // plan only, tensor cores off on every rank (replicated cell count)
+    for (auto& v : ws.tc_local) v = 0;
+    return EGGSYNC_OK;
+  }
   if (hi <= lo) return EGGSYNC_OK;
-  if (tc_enabled(ws, D)) return run_update_tc<D>(ws, lo, hi, nbr);
   return run_update_simt<D>(ws, lo, hi, nbr);
 }
 

@@ -55,6 +55,7 @@ class TorchComm:
         import torch.distributed as dist
         self.torch, self.dist, self.group, self.mode = torch, dist, group, mode
         self.device = torch.device(device)
+        self.backend = dist.get_backend(group)
         self.world = dist.get_world_size(group)
         self.rank = dist.get_rank(group)
         span = math.ceil(n / self.world)
@@ -74,13 +75,26 @@ class TorchComm:
         self.flag = torch.zeros(1, dtype=torch.int32, device=device)
 
     def reduce_min(self, v: int) -> int:
-        self.flag.fill_(int(v))
-        self.dist.all_reduce(self.flag, op=self.dist.ReduceOp.MIN, group=self.group)
-        return int(self.flag.item())
+        flag = self.flag if self.backend == "nccl" or self.device.type != "cuda" else self.flag.cpu()
+        flag.fill_(int(v))
+        self.dist.all_reduce(flag, op=self.dist.ReduceOp.MIN, group=self.group)
+        return int(flag.item())
+
+    def reduce_plan(self, stats):
+        """SUM of the entry / point / tile counts, MAX of the flags (eggsync.h)."""
+        torch = self.torch
+        dev = self.device if self.device.type == "cuda" and self.backend == "nccl" else torch.device("cpu")
+        t = torch.tensor(stats, dtype=torch.int64, device=dev)
+        s, m = t[:3].clone(), t[3:].clone()
+        self.dist.all_reduce(s, op=self.dist.ReduceOp.SUM, group=self.group)
+        self.dist.all_reduce(m, op=self.dist.ReduceOp.MAX, group=self.group)
+        return torch.cat([s, m]).cpu().numpy()
 
     def update(self, ctx) -> None:
         if self.mode == "interleaved":
-            ctx.update_owned(self.rank, self.world)
+            # the update kernel is chosen from plan statistics of all ranks, as one GPU would
+            g = self.reduce_plan(ctx.plan_owned(self.rank, self.world))
+            ctx.update_planned(self.rank, self.world, g)
         else:
             ctx.update(self.lo, self.hi)
 
@@ -96,7 +110,13 @@ class TorchComm:
             ctx.pack_into(self.lo, self.cnt, self.send)
         if cuda:
             cs.wait_stream(xs)   # the all-gather reads `send` after the pack kernel
-        self.dist.all_gather_into_tensor(self.recv, self.send, group=self.group)
+        if cuda and self.backend != "nccl":
+            # gloo between processes that share a GPU (tests): stage the exchange through host memory
+            recv = torch.empty(self.recv.shape, dtype=self.recv.dtype)
+            self.dist.all_gather_into_tensor(recv, self.send.cpu(), group=self.group)
+            self.recv.copy_(recv)
+        else:
+            self.dist.all_gather_into_tensor(self.recv, self.send, group=self.group)
         if cuda:
             xs.wait_stream(cs)   # the unpack kernel reads `recv` after the all-gather
         view = self.recv.view(self.world, -1, self.cnt)

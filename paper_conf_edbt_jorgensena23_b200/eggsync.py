@@ -27,7 +27,8 @@ SYMBOLS = [
     "eggsync_ctx_unpack", "eggsync_ctx_advance", "eggsync_ctx_labels", "eggsync_ctx_coords",
     "eggsync_ctx_run", "eggsync_ctx_stream", "eggsync_ctx_work", "eggsync_ctx_tc_work", "eggsync_ctx_launches",
     "eggsync_release_cache", "eggsync_ctx_update_owned", "eggsync_ctx_owned_count", "eggsync_ctx_pack_owned",
-    "eggsync_ctx_unpack_owned", "eggsync_sync_step", "eggsync_sync_lambda",
+    "eggsync_ctx_unpack_owned", "eggsync_ctx_plan_owned", "eggsync_ctx_update_planned", "eggsync_sync_step",
+    "eggsync_sync_lambda",
 ]
 
 
@@ -99,6 +100,8 @@ def lib():
             "eggsync_ctx_owned_count": ([vp, i32], ctypes.c_int64),
             "eggsync_ctx_pack_owned": ([vp, i32, i32, vp], ctypes.c_int),
             "eggsync_ctx_unpack_owned": ([vp, vp, i32], ctypes.c_int),
+            "eggsync_ctx_plan_owned": ([vp, i32, i32, vp], ctypes.c_int),
+            "eggsync_ctx_update_planned": ([vp, i32, i32, vp], ctypes.c_int),
             "eggsync_sync_step": ([vp, i64, i32, f32, i32, vp, vp], ctypes.c_int),
             "eggsync_sync_lambda": ([vp, i64, i32, f32, ctypes.c_double, i32, i32, vp, vp], ctypes.c_int),
         }
@@ -351,6 +354,17 @@ class Context:
 
     def pack_owned_into(self, rank: int, ranks: int, tensor):
         _check(lib().eggsync_ctx_pack_owned(self.h, rank, ranks, ctypes.c_void_p(tensor.data_ptr())))
+
+    def plan_owned(self, rank: int, ranks: int):
+        """Plan pass of the owned tiles; returns int64[6] statistics (see eggsync.h)."""
+        out = np.zeros(6, np.int64)
+        _check(lib().eggsync_ctx_plan_owned(self.h, rank, ranks, out.ctypes.data_as(ctypes.c_void_p)))
+        return out
+
+    def update_planned(self, rank: int, ranks: int, global_stats):
+        """Update of the owned tiles with the kernel chosen from rank-reduced plan statistics."""
+        g = np.ascontiguousarray(global_stats, dtype=np.int64)
+        _check(lib().eggsync_ctx_update_planned(self.h, rank, ranks, g.ctypes.data_as(ctypes.c_void_p)))
 
     def unpack_owned_from(self, tensor, ranks: int):
         _check(lib().eggsync_ctx_unpack_owned(self.h, ctypes.c_void_p(tensor.data_ptr()), ranks))

@@ -82,6 +82,15 @@ class OracleCtx:
         k = np.arange(cnt)
         return ((k // self.B) * R + r) * self.B + k % self.B
 
+    def plan_owned(self, r, R):  # the library's plan statistics: [entries, points, tiles, overflow, max cell, tc]
+        return np.array([7 * (r + 1), 7 * (r + 1), r + 1, 0, 3, 1], np.int64)
+
+    def update_planned(self, r, R, g):
+        # every rank sees the same rank-reduced statistics (SUM of 0..2, MAX of 3..5)
+        tot = sum(range(1, R + 1))
+        assert list(g) == [7 * tot, 7 * tot, tot, 0, 3, 1], g
+        self.update_owned(r, R)
+
     def update_owned(self, r, R):
         pos = self._owned_pos(r, R, self.owned_count(R))
         pos = pos[pos < self.n]
