@@ -111,7 +111,12 @@ void eggsync_default_opts(eggsync_opts *o);
 int eggsync_cluster(const float *points, int64_t n, int32_t d, float eps, int32_t *labels_out,
                     int32_t *iters_out);
 
-/* As eggsync_cluster with options (device pointers, stream, stats, coords_out, max_iters). */
+/* As eggsync_cluster with options (device pointers, stream, stats, coords_out, max_iters).
+ * Small inputs (n <= 4096, n*d <= 8192, d <= 8, the cell key in 64 bits, GRID mode, no
+ * stats requested) run Algorithm 4 (L258-278) in ONE kernel launch -- a 16-CTA thread-block
+ * cluster holding the state in distributed shared memory, no per-iteration host round trip
+ * (SURVEY.md §8(f) F1); the same readings and results as the grid path (environment
+ * EGGSYNC_SMALL=0 forces the grid path). */
 int eggsync_cluster_ex(const float *points, int64_t n, int32_t d, float eps, const eggsync_opts *opts,
                        int32_t *labels_out, int32_t *iters_out);
 

@@ -586,7 +586,11 @@ extern "C" {
 const char* eggsync_last_error(void) { return g_err.c_str(); }
 const char* eggsync_version(void) { return "eggsync-b200 0.1 (sm_100a)"; }
 
-void eggsync_release_cache(void) { cache_clear(); }
+static void small_release();  // the one-launch path's scratch (below)
+void eggsync_release_cache(void) {
+  cache_clear();
+  small_release();
+}
 
 void eggsync_default_opts(eggsync_opts* o) {
   if (!o) return;
@@ -621,6 +625,81 @@ static int get_opts(const eggsync_opts* in, eggsync_opts* o) {
   return EGGSYNC_OK;
 }
 
+// ------------------------------------------------------------------ small inputs (F1)
+// Scratch of the one-launch path, cached per device (grow-only): input, labels, coordinates,
+// [iterations, converged] -- so that a small clustering costs one H2D, one launch, one D2H.
+struct SmallScratch {
+  int device = -1;
+  char* dev = nullptr;
+  size_t bytes = 0;
+  char* host = nullptr;  // pinned mirror of the outputs
+  size_t hbytes = 0;
+};
+static std::mutex g_small_mu;
+static std::vector<SmallScratch> g_small;
+
+static void small_release() {
+  std::lock_guard<std::mutex> lk(g_small_mu);
+  for (auto& c : g_small) {
+    cudaSetDevice(c.device);
+    if (c.dev) cudaFree(c.dev);
+    if (c.host) cudaFreeHost(c.host);
+  }
+  g_small.clear();
+}
+
+static int small_path(const float* points, int64_t n, int32_t d, const Consts& k, const eggsync_opts& o,
+                      int32_t* labels_out, int32_t* iters_out, int* rc_out) {
+  int dev = 0;
+  EGG_CUDA(cudaGetDevice(&dev));
+  const size_t nx = (size_t)n * d * sizeof(float), nl = (size_t)n * sizeof(int32_t);
+  const size_t need = 2 * nx + nl + 64;
+  std::lock_guard<std::mutex> lk(g_small_mu);
+  SmallScratch* sc = nullptr;
+  for (auto& c : g_small)
+    if (c.device == dev) sc = &c;
+  if (!sc) {
+    g_small.push_back(SmallScratch{});
+    sc = &g_small.back();
+    sc->device = dev;
+  }
+  if (sc->bytes < need) {
+    if (sc->dev) cudaFree(sc->dev);
+    sc->bytes = 0;
+    EGG_CUDA(cudaMalloc((void**)&sc->dev, need));
+    sc->bytes = need;
+  }
+  if (sc->hbytes < need) {
+    if (sc->host) cudaFreeHost(sc->host);
+    sc->hbytes = 0;
+    EGG_CUDA(cudaMallocHost((void**)&sc->host, need));
+    sc->hbytes = need;
+  }
+  cudaStream_t st = (cudaStream_t)o.stream;
+  float* x = reinterpret_cast<float*>(sc->dev);
+  float* co = reinterpret_cast<float*>(sc->dev + nx);
+  int32_t* lab = reinterpret_cast<int32_t*>(sc->dev + 2 * nx);
+  int32_t* out = reinterpret_cast<int32_t*>(sc->dev + 2 * nx + nl);
+  const float* src = points;
+  if (!o.device_pointers) {
+    EGG_CUDA(cudaMemcpyAsync(x, points, nx, cudaMemcpyHostToDevice, st));
+    src = x;
+  }
+  EGG_TRY(small_cluster(src, n, d, k, o.max_iters, o.device_pointers ? labels_out : lab,
+                        o.device_pointers && o.coords_out ? o.coords_out : co, out, st));
+  EGG_CUDA(cudaGetLastError());
+  int32_t* hout = reinterpret_cast<int32_t*>(sc->host);
+  EGG_CUDA(cudaMemcpyAsync(hout, out, 2 * sizeof(int32_t), cudaMemcpyDeviceToHost, st));
+  if (!o.device_pointers) {
+    EGG_CUDA(cudaMemcpyAsync(labels_out, lab, nl, cudaMemcpyDeviceToHost, st));
+    if (o.coords_out) EGG_CUDA(cudaMemcpyAsync(o.coords_out, co, nx, cudaMemcpyDeviceToHost, st));
+  }
+  EGG_CUDA(cudaStreamSynchronize(st));
+  *iters_out = hout[0];
+  *rc_out = hout[1] ? EGGSYNC_OK : EGGSYNC_NOT_CONVERGED;
+  return EGGSYNC_OK;
+}
+
 int eggsync_cluster_ex(const float* points, int64_t n, int32_t d, float eps, const eggsync_opts* opts,
                        int32_t* labels_out, int32_t* iters_out) {
   eggsync_opts o;
@@ -634,6 +713,24 @@ int eggsync_cluster_ex(const float* points, int64_t n, int32_t d, float eps, con
   DeviceGuard g;
   EGG_TRY(g.set(o.device));
   if (o.term_mode == EGGSYNC_TERM_DEF42) return def42_cluster(points, n, d, eps, o, labels_out, iters_out);
+  {
+    // F1: small inputs run Algorithm 4 in one kernel launch (no per-iteration host round trip);
+    // validation of the domain happens inside (a point outside [0,1] is rejected below first)
+    Consts kc;
+    std::string why;
+    if (!o.stats && make_consts(n, d, eps, &kc, &why, o.cw_factor) && small_eligible(n, d, kc)) {
+      if (!o.device_pointers) {  // EDOMAIN before any output is written (host input)
+        for (int64_t t = 0; t < n * d; ++t)
+          if (!(points[t] >= 0.f && points[t] <= 1.f)) {
+            set_error("a coordinate is NaN/Inf or outside [0,1] (PAPER.md L70: data must be normalised)");
+            return EGGSYNC_EDOMAIN;
+          }
+        int rc = EGGSYNC_OK;
+        EGG_TRY(small_path(points, n, d, kc, o, labels_out, iters_out, &rc));
+        return rc;
+      }
+    }
+  }
   eggsync_stats local{};
   eggsync_stats* stats = o.stats ? &local : nullptr;
   auto t0 = std::chrono::steady_clock::now();

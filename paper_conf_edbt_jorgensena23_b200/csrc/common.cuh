@@ -96,6 +96,11 @@ struct Consts {
 
 bool make_consts(int64_t n, int d, float eps, Consts* c, std::string* why, double cw_factor = 1.0);
 
+// F1 one-launch clustering of small inputs (small.cu)
+bool small_eligible(int64_t n, int d, const Consts& k);
+int small_cluster(const float* x_dev, int64_t n, int d, const Consts& k, int32_t max_iters, int32_t* labels_dev,
+                  float* coords_dev, int32_t* out_dev, cudaStream_t st);
+
 // term_mode = EGGSYNC_TERM_DEF42 clustering on the direct kernels (sync_brute.cu).
 int def42_cluster(const float* points, int64_t n, int d, float eps, const eggsync_opts& o, int32_t* labels_out,
                   int32_t* iters_out);

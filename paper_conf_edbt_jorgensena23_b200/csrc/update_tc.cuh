@@ -211,87 +211,117 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
     for (int k = 0; k < kP; ++k) stk[1 + k] = (int)am[k];
   }
   __syncwarp();
+  // Two stack entries per step: their node data (box, meta, count) are loaded together, so
+  // the walk's dependent global-load chain is half as long (the order of the entries within
+  // a tile is immaterial: the update's sums are exact integers).
   int sp = 1;
   while (sp > 0) {
-    --sp;
-    const int node = stk[sp * 8];
-    uint32_t m[kP];
+    const int nb = sp >= 2 ? 2 : 1;
+    int nodes[2];
+    uint32_t mk[2][kP];
 #pragma unroll
-    for (int k = 0; k < kP; ++k) m[k] = (uint32_t)stk[sp * 8 + 1 + k];
+    for (int b = 0; b < 2; ++b) {
+      const int e = b < nb ? sp - 1 - b : sp - 1;
+      nodes[b] = stk[e * 8];
+#pragma unroll
+      for (int k = 0; k < kP; ++k) mk[b][k] = (uint32_t)stk[e * 8 + 1 + k];
+    }
+    sp -= nb;
     __syncwarp();
-    if (node & (int)kLeafBit) {  // a single cell: always an entry
-      push(node & 0x7fffffff, 1, a.c_cnt[node & 0x7fffffff]);
-      continue;
+    float4 bx[2][BS / 4];
+    int4 meta[2];
+    int tcn[2];
+#pragma unroll
+    for (int b = 0; b < 2; ++b) {
+      const int nd = nodes[b] & 0x7fffffff;
+      const bool internal = b < nb && !(nodes[b] & (int)kLeafBit);
+      const float4* __restrict__ src = reinterpret_cast<const float4*>(a.t_box + (int64_t)(internal ? nd : 0) * BS);
+#pragma unroll
+      for (int k = 0; k < BS / 4; ++k) bx[b][k] = src[k];
+      meta[b] = a.t_meta[internal ? nd : 0];
+      tcn[b] = internal ? a.t_cnt[nd] : (b < nb ? a.c_cnt[nd] : 0);
     }
-    const float* __restrict__ bx = a.t_box + (int64_t)node * BS;
-    float m0[kP], x0[kP];
+    bool overflow = false;
 #pragma unroll
-    for (int k = 0; k < kP; ++k) m0[k] = x0[k] = 0.f;
-#pragma unroll
-    for (int i = 0; i < D; ++i) {
-      const float blo = bx[i] - ov[i], bhi = bx[D + i] - ov[i];
-#pragma unroll
-      for (int k = 0; k < kP; ++k) {
-        const float dl = blo - q[k][i], dh = q[k][i] - bhi;
-        const float mn = fmaxf(fmaxf(dl, dh), 0.f), mx = fmaxf(-dl, -dh);
-        m0[k] = fmaf(mn, mn, m0[k]);
-        x0[k] = fmaf(mx, mx, x0[k]);
+    for (int b = 0; b < 2; ++b) {
+      if (b >= nb) break;
+      const int node = nodes[b];
+      if (node & (int)kLeafBit) {  // a single cell: always an entry
+        push(node & 0x7fffffff, 1, tcn[b]);
+        continue;
       }
-    }
-    bool full[kP], part[kP];
-    uint32_t pm[kP], fm[kP];
-    bool any_part = false;
+      const float* bxf = reinterpret_cast<const float*>(bx[b]);
+      float m0[kP], x0[kP];
 #pragma unroll
-    for (int k = 0; k < kP; ++k) {
-      const bool act = (m[k] >> lane) & 1u;
-      full[k] = act && x0[k] <= lim_full;
-      part[k] = act && !full[k] && m0[k] <= lim_out;
-      pm[k] = __ballot_sync(FULLMASK, part[k]);
-      fm[k] = __ballot_sync(FULLMASK, full[k]);
-      any_part |= pm[k] != 0u;
-    }
-    if (!any_part) {  // nobody needs to look inside: full points take the subtree summary
-      bool anyf = false;
+      for (int k = 0; k < kP; ++k) m0[k] = x0[k] = 0.f;
 #pragma unroll
-      for (int k = 0; k < kP; ++k) anyf |= fm[k] != 0u;
-      if (anyf) {
-        const int cnt = a.t_cnt[node];
-        const float* __restrict__ sm = a.t_sum + (int64_t)node * BS;
+      for (int i = 0; i < D; ++i) {
+        const float blo = bxf[i] - ov[i], bhi = bxf[D + i] - ov[i];
 #pragma unroll
         for (int k = 0; k < kP; ++k) {
-          if (full[k]) {
-            N[k] += cnt;
-#pragma unroll
-            for (int i = 0; i < 2 * D; ++i) {
-              double* dst = a.full_S + (int64_t)i * a.n + j[k];
-              *dst = (touched[k] ? *dst : 0.0) + (double)sm[i];
-            }
-            touched[k] = true;
-          }
+          const float dl = blo - q[k][i], dh = q[k][i] - bhi;
+          const float mn = fmaxf(fmaxf(dl, dh), 0.f), mx = fmaxf(-dl, -dh);
+          m0[k] = fmaf(mn, mn, m0[k]);
+          x0[k] = fmaf(mx, mx, x0[k]);
         }
       }
-      continue;
+      bool full[kP];
+      uint32_t pm[kP], fm[kP];
+      bool any_part = false;
+#pragma unroll
+      for (int k = 0; k < kP; ++k) {
+        const bool act = (mk[b][k] >> lane) & 1u;
+        full[k] = act && x0[k] <= lim_full;
+        const bool part = act && !full[k] && m0[k] <= lim_out;
+        pm[k] = __ballot_sync(FULLMASK, part);
+        fm[k] = __ballot_sync(FULLMASK, full[k]);
+        any_part |= pm[k] != 0u;
+      }
+      if (!any_part) {  // nobody needs to look inside: full points take the subtree summary
+        bool anyf = false;
+#pragma unroll
+        for (int k = 0; k < kP; ++k) anyf |= fm[k] != 0u;
+        if (anyf) {
+          const float* __restrict__ sm = a.t_sum + (int64_t)node * BS;
+#pragma unroll
+          for (int k = 0; k < kP; ++k) {
+            if (full[k]) {
+              N[k] += tcn[b];
+#pragma unroll
+              for (int i = 0; i < 2 * D; ++i) {
+                double* dst = a.full_S + (int64_t)i * a.n + j[k];
+                *dst = (touched[k] ? *dst : 0.0) + (double)sm[i];
+              }
+              touched[k] = true;
+            }
+          }
+        }
+        continue;
+      }
+      const int ncell = meta[b].y - meta[b].x + 1;
+      if (ncell <= a.bucket) {
+        push(meta[b].x, ncell, tcn[b]);
+        continue;
+      }
+      if (sp + 2 > a.stack_len) {
+        overflow = true;
+        break;
+      }
+      if (lane == 0) {
+        stk[sp * 8] = meta[b].w;
+        stk[(sp + 1) * 8] = meta[b].z;
+#pragma unroll
+        for (int k = 0; k < kP; ++k) {
+          stk[sp * 8 + 1 + k] = (int)(pm[k] | fm[k]);
+          stk[(sp + 1) * 8 + 1 + k] = (int)(pm[k] | fm[k]);
+        }
+      }
+      sp += 2;
     }
-    const int4 meta = a.t_meta[node];
-    const int ncell = meta.y - meta.x + 1;
-    if (ncell <= a.bucket) {
-      push(meta.x, ncell, a.t_cnt[node]);
-      continue;
-    }
-    if (sp + 2 > a.stack_len) {
+    if (overflow) {
       if (lane == 0) atomicExch(&a.flags[3], 1);
       break;
     }
-    if (lane == 0) {
-      stk[sp * 8] = meta.w;
-      stk[(sp + 1) * 8] = meta.z;
-#pragma unroll
-      for (int k = 0; k < kP; ++k) {
-        stk[sp * 8 + 1 + k] = (int)(pm[k] | fm[k]);
-        stk[(sp + 1) * 8 + 1 + k] = (int)(pm[k] | fm[k]);
-      }
-    }
-    sp += 2;
     __syncwarp();
   }
   if (lane == 0) {
