@@ -340,6 +340,72 @@ def run_ours(args):
         dist.destroy_process_group()
 
 
+# ------------------------------------------------- E2: sharded points (C5)
+def run_shard(args):
+    """--shard: SURVEY.md §8(e) E2 -- no rank holds all points (slab shards + halo exchange,
+    distributed.run_sharded); one step = one complete clustering.  Device time (CUDA events
+    on the current stream, barrier on both sides), max over ranks."""
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_edbt_jorgensena23_b200 import datagen, distributed as DR, eggsync as E
+
+    world, rank, local = dist_env()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    dist.init_process_group("nccl" if world > 1 else "gloo", device_id=dev if world > 1 else None,
+                            **({} if world > 1 else {"rank": 0, "world_size": 1,
+                                                     "init_method": "tcp://127.0.0.1:%d" % _free_port()}))
+    c = datagen.make_config(args.config)
+    X = c.generate(args.seed)
+    n, d = X.shape
+    share = np.array_split(np.arange(n), world)[rank]
+    stream = torch.cuda.Stream(dev)
+    torch.cuda.set_stream(stream)
+    Xd = torch.from_numpy(X[share]).to(dev)
+    gd = torch.from_numpy(share.astype(np.int64)).to(dev)
+    ex = DR.ShardExchange(d, c.eps, dev)
+    make = lambda m, dd: E.Context(m, dd, c.eps, device=local, stream=stream.cuda_stream)  # noqa: E731
+
+    def one():
+        return DR.run_sharded(Xd, gd, c.eps, ex, make)
+
+    for _ in range(args.warmup):
+        it, ok, lab, _ = one()
+    ms = []
+    dist.barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        for _ in range(args.steps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            it, ok, lab, _ = one()
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ms.append(e0.elapsed_time(e1))
+    dist.barrier()
+    t = torch.tensor([statistics.mean(ms)], dtype=torch.float64, device=dev if world > 1 else "cpu")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    msv = float(t[0])
+    if rank == 0:
+        print(json.dumps({
+            "metric": METRIC, "value": n * it / (msv / 1e3), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": msv, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {"workload": workload_desc(c), "n": n, "d": d, "eps": c.eps, "iters": it, "converged": ok,
+                       "clusters": int(lab.max()) + 1, "parallelism": f"E2 sharded points: slab shards + halo x{world}",
+                       "l2": "inputs resident in HBM (n*d*4 B per rank share); no flush (whole clusterings)"},
+            "clocks": clk.summary(), "gpu_launches": None}), flush=True)
+    dist.destroy_process_group()
+
+
+def _free_port():
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        return sk.getsockname()[1]
+
+
 # ---------------------------------------------------- reference arm (oracle)
 def run_reference(args):
     world, rank, _ = dist_env()
@@ -400,6 +466,7 @@ def main():
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-direct", action="store_true", help="skip the direct-path (GPU-SynC-style) context timing")
+    ap.add_argument("--shard", action="store_true", help="E2: sharded points (slab shards + halo), e.g. --config C5")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
@@ -410,6 +477,8 @@ def main():
         sys.exit(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={world}; launch one rank per GPU")
     if args.impl == "reference":
         run_reference(args)
+    elif args.shard:
+        run_shard(args)
     else:
         run_ours(args)
 

@@ -251,6 +251,13 @@ int64_t eggsync_ctx_owned_count(eggsync_ctx *ctx, int32_t ranks);
 int eggsync_ctx_pack_owned(eggsync_ctx *ctx, int32_t rank, int32_t ranks, float *buf);
 int eggsync_ctx_unpack_owned(eggsync_ctx *ctx, const float *gathered, int32_t ranks);
 
+/* Sharded runs (distributed.run_sharded): the context holds a rank's own
+ * points -- the first n_own of the loaded points -- followed by its halo (the other ranks'
+ * points within eps+delta of the own ones).  Every point is updated, but only own points
+ * contribute to the criterion flags (first term in the update, second term).  n_own >= n
+ * (the default) means all points are own.  Errors: EINVAL. */
+int eggsync_ctx_set_own(eggsync_ctx *ctx, int64_t n_own);
+
 /* Collective choice of the update kernel (tensor-core or SIMT) for a multi-rank update, so
  * that every rank -- and one GPU running the whole range -- choose alike and the result stays
  * bitwise identical to one GPU.  eggsync_ctx_plan_owned runs the tensor-core plan pass

@@ -1072,6 +1072,12 @@ int eggsync_ctx_update_planned(eggsync_ctx* ctx, int32_t rank, int32_t ranks, co
   return rc;
 }
 
+int eggsync_ctx_set_own(eggsync_ctx* ctx, int64_t n_own) {
+  if (!ctx || n_own < 0) return EGGSYNC_EINVAL;
+  ctx->ws.n_own = n_own >= ctx->ws.n ? INT64_MAX : n_own;
+  return EGGSYNC_OK;
+}
+
 int64_t eggsync_ctx_owned_count(eggsync_ctx* ctx, int32_t ranks) {
   if (!ctx || ranks < 1) return -1;
   return owned_count(ctx->ws, ranks);

@@ -244,6 +244,10 @@ struct Workspace {
   bool count_work = false;
   int64_t launches = 0;  // kernel launches issued on this workspace (CUB internals counted by pass)
   int32_t own_stride = 1, own_offset = 0;  // block-interleaved ownership of the next update
+  // sharded multi-rank runs (E2): the context holds a rank's own points (original local index
+  // < n_own) followed by its halo; only own points contribute to the criterion flags
+  int64_t n_own = INT64_MAX;
+  const uint32_t* own_orig() const { return n_own < n ? orig[ocur] : nullptr; }
   // tensor-core update (update_tc.cuh): plan-pass outputs
   double* full_S = nullptr;     // [2d][n] per-point sums of subtrees added whole (sorted order)
   int32_t* full_N = nullptr;    // [n]

@@ -14,6 +14,8 @@ namespace egg {
 
 template <int D>
 struct TermArgs {
+  const uint32_t* __restrict__ orig;  // sharded runs: original local index (own iff < n_own), else nullptr
+  int64_t n_own;
   const float* __restrict__ xs;
   const int32_t* __restrict__ g_of;    // grid cell of each sorted point
   const int32_t* __restrict__ u2co;    // unit -> grid cell (nullptr: identity)
@@ -54,7 +56,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_second(const TermArgs<D> 
   const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
   int2* stk = reinterpret_cast<int2*>(smem) + wid * a.stack_len;
   const int64_t j = a.lo + ((int64_t)blockIdx.x * kWarpsPerCta + wid) * 32 + lane;
-  const bool valid = j < a.hi;
+  const bool valid = j < a.hi && (!a.orig || a.orig[j] < (uint32_t)a.n_own);  // halo points do not test
   const unsigned amask = __ballot_sync(FULLMASK, valid);
   if (amask == 0u) return;
   float p[D];
@@ -179,6 +181,8 @@ template <int D>
 int run_second_term(Workspace& ws, int64_t lo, int64_t hi) {
   if (hi <= lo) return EGGSYNC_OK;
   TermArgs<D> a;
+  a.orig = ws.own_orig();
+  a.n_own = ws.n_own;
   a.xs = ws.xs[ws.xcur];
   a.g_of = ws.g_of;
   a.u2co = ws.g_u2co;

@@ -67,6 +67,8 @@ struct PPL {
 
 template <int D>
 struct UpdArgs {
+  const uint32_t* __restrict__ orig;  // sharded runs: original local index (own iff < n_own), else nullptr
+  int64_t n_own;
   const float* __restrict__ xs;  // D^t, SoA [D][n], sorted
   float* __restrict__ xs_next;   // D^{t+1}, SoA [D][n], sorted
   const float* __restrict__ sn;  // sin(x), SoA [D][n]
@@ -658,9 +660,12 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(cons
         sincos(x, &sx, &cx);
         const double Sd = mst[(k * 2 * D + i) * 32 + lane], Cd = mst[(k * 2 * D + D + i) * 32 + lane];
         const double xn = x + (cx * Sd - sx * Cd) * inv;  // Eq.5
+        // x' lies in the range of N(p) (L104) and so in [0,1]; rounding of the summaries can put
+        // it an ulp outside, which the clamp removes (the state stays in the domain, L70)
         a.xs_next[(int64_t)i * a.n + L.j[k]] = fminf(fmaxf((float)xn, 0.f), 1.f);
       }
-      f1 = f1 && (L.N[k] == a.g_cnt[a.g_of[L.j[k]]]);  // Alg 3 l.14-15 (L248)
+      const bool own = !a.orig || a.orig[L.j[k]] < (uint32_t)a.n_own;
+      f1 = f1 && (!own || L.N[k] == a.g_cnt[a.g_of[L.j[k]]]);  // Alg 3 l.14-15 (L248)
       if (a.nbr) a.nbr[L.j[k]] = L.N[k];
     }
   }
@@ -683,6 +688,8 @@ template <int D>
 int run_update_simt(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   if (hi <= lo) return EGGSYNC_OK;
   UpdArgs<D> a;
+  a.orig = ws.own_orig();
+  a.n_own = ws.n_own;
   a.xs = ws.xs[ws.xcur];
   a.xs_next = ws.xs[ws.xcur ^ 1];
   a.sn = ws.sn;

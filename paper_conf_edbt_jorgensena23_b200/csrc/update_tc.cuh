@@ -388,6 +388,8 @@ __global__ void __launch_bounds__(128) k_tc_expand(const int2* __restrict__ rang
 // ----------------------------------------------------------------------------------------
 template <int D>
 struct TcArgs {
+  const uint32_t* __restrict__ orig;  // sharded runs: original local index (own iff < n_own), else nullptr
+  int64_t n_own;
   const float* __restrict__ xs;
   float* __restrict__ xs_next;
   const float* __restrict__ sn;
@@ -1037,10 +1039,12 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
         const double x = (double)pe[i];
         sincos(x, &sx, &cx);
         const double xn = x + (cx * S - sx * Cc) * inv;  // Eq.5
-        a.xs_next[(int64_t)i * a.n + j] = (float)xn;
+        // x' lies in the range of N(p) (L104) and so in [0,1]; the 2^-21 fixed point of the
+        // summaries can put it an ulp or two outside, which the clamp removes (domain, L70)
+        a.xs_next[(int64_t)i * a.n + j] = fminf(fmaxf((float)xn, 0.f), 1.f);
       }
       const bool f1 = Ni == (int64_t)a.g_cnt[a.g_of[j]];  // Alg 3 l.14-15 (L248)
-      if (!f1) atomicAnd(&a.flags[0], 0);
+      if (!f1 && (!a.orig || a.orig[j] < (uint32_t)a.n_own)) atomicAnd(&a.flags[0], 0);
       if (a.nbr) a.nbr[j] = (int32_t)Ni;
     }
   }
@@ -1226,6 +1230,8 @@ int run_planned_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr, int64_t 
     const size_t smem = (size_t)nst * sbytes + C::kFixedBytes;
 
     TcArgs<D> a;
+    a.orig = ws.own_orig();
+    a.n_own = ws.n_own;
     a.xs = ws.xs[ws.xcur];
     a.xs_next = ws.xs[ws.xcur ^ 1];
     a.sn = ws.sn;

@@ -159,3 +159,172 @@ def run(ctx, comm=None, max_iters: int = 10000, hooks=None):
     if not synced:
         labels = ctx.labels()
     return t, synced, labels
+
+
+# --------------------------------------------------------------------------------------
+# E2: sharded points.  No rank holds all n points: each rank owns the
+# points of one slab of the first coordinate (quantile splitters, rebalanced every
+# iteration) and receives a halo -- the other ranks' points within HALO * eps of its slab.
+# With HALO >= 1.5 + delta/eps every grid cell that matters for an own point is complete
+# locally: a cell within eps(+delta) of an own point has all its points within eps/2 more
+# (cell diagonal eps/2, L252), so the own points' neighbourhoods (Eq.1), their cells
+# (first term, L248/L252) and the cells of their shell points (MBR(N_eps/2(q)) of the
+# second term, L108-110) are exact; only the own points' criterion flags count
+# (eggsync_ctx_set_own).  Per iteration: one all-to-all moving points to their owners plus
+# halo copies, a local build + update on own + halo, MIN all-reduces of the flags.  The
+# labels are the cells of the verified state, gathered to rank 0 and numbered there by the
+# library (L256, R14).  Local trees differ from one GPU's, so the sums are summed in another
+# order: results agree with one GPU within the parity tolerance, not bitwise.
+# --------------------------------------------------------------------------------------
+HALO = 1.6
+
+
+class ShardExchange:
+    """Data distribution of the sharded driver (torch.distributed plumbing only)."""
+
+    def __init__(self, d: int, eps: float, device, group=None, sample: int = 4096):
+        import torch
+        import torch.distributed as dist
+        self.torch, self.dist, self.group = torch, dist, group
+        self.world = dist.get_world_size(group)
+        self.rank = dist.get_rank(group)
+        self.device = torch.device(device)
+        self.backend = dist.get_backend(group)
+        self.d, self.h, self.sample = d, HALO * float(eps), sample
+
+    def _coll_dev(self):
+        return self.device if (self.backend == "nccl" and self.device.type == "cuda") else self.torch.device("cpu")
+
+    def _all_gather_1d(self, t):
+        torch = self.torch
+        dev = self._coll_dev()
+        n = torch.tensor([t.numel()], dtype=torch.int64, device=dev)
+        ns = [torch.zeros_like(n) for _ in range(self.world)]
+        self.dist.all_gather(ns, n, group=self.group)
+        m = int(max(int(x) for x in ns))
+        buf = torch.zeros(m, dtype=t.dtype, device=dev)
+        buf[: t.numel()] = t.to(dev)
+        outs = [torch.zeros_like(buf) for _ in range(self.world)]
+        self.dist.all_gather(outs, buf, group=self.group)
+        return torch.cat([o[: int(k)] for o, k in zip(outs, ns)])
+
+    def splitters(self, x0):
+        """World-1 quantiles of the first coordinate over a sample of every rank's points."""
+        torch = self.torch
+        k = min(self.sample, x0.numel())
+        idx = torch.linspace(0, max(x0.numel() - 1, 0), k, device=x0.device).long() if k else \
+            torch.zeros(0, dtype=torch.long, device=x0.device)
+        allx = self._all_gather_1d(torch.sort(x0)[0][idx].float()).sort()[0]
+        if allx.numel() == 0:
+            return torch.zeros(self.world - 1, device=x0.device)
+        q = torch.linspace(0, allx.numel() - 1, self.world + 1)[1:-1].round().long()
+        return allx[q.to(allx.device)].to(x0.device)
+
+    def exchange(self, X, gid, split):
+        """Own points to their slab owners and halo copies to every rank within self.h of them.
+        Returns (own X, own gid, halo X, halo gid) on this rank."""
+        torch = self.torch
+        R, dev = self.world, X.device
+        x0 = X[:, 0]
+        lo = torch.cat([torch.full((1,), -1e30, device=dev), split.to(dev)])
+        hi = torch.cat([split.to(dev), torch.full((1,), 1e30, device=dev)])
+        owner = torch.searchsorted(split.to(dev).contiguous(), x0.contiguous(), right=True)
+        parts, counts = [], []
+        for r in range(R):
+            own = owner == r
+            halo = (~own) & (x0 >= lo[r] - self.h) & (x0 < hi[r] + self.h)
+            for m in (own, halo):
+                parts.append((X[m], gid[m]))
+                counts.append(int(m.sum()))
+        cnt = torch.tensor(counts, dtype=torch.int64, device=self._coll_dev())
+        rcnt = torch.empty_like(cnt)
+        self.dist.all_to_all_single(rcnt, cnt, group=self.group)
+        send_x = torch.cat([p[0] for p in parts]).reshape(-1)
+        send_g = torch.cat([p[1] for p in parts])
+        ssz = [counts[2 * r] + counts[2 * r + 1] for r in range(R)]
+        rc = rcnt.cpu().tolist()
+        rsz = [rc[2 * r] + rc[2 * r + 1] for r in range(R)]
+        cd = self._coll_dev()
+        recv_x = torch.empty(sum(rsz) * self.d, dtype=X.dtype, device=cd)
+        recv_g = torch.empty(sum(rsz), dtype=gid.dtype, device=cd)
+        self.dist.all_to_all_single(recv_x, send_x.to(cd), [s * self.d for s in rsz], [s * self.d for s in ssz],
+                                    group=self.group)
+        self.dist.all_to_all_single(recv_g, send_g.to(cd), rsz, ssz, group=self.group)
+        recv_x = recv_x.to(dev).reshape(-1, self.d)
+        recv_g = recv_g.to(dev)
+        own_m = torch.zeros(sum(rsz), dtype=torch.bool, device=dev)
+        off = 0
+        for r in range(R):
+            own_m[off: off + rc[2 * r]] = True
+            off += rsz[r]
+        return recv_x[own_m], recv_g[own_m], recv_x[~own_m], recv_g[~own_m]
+
+    def min(self, v: int) -> int:
+        t = self.torch.tensor([int(v)], dtype=self.torch.int32, device=self._coll_dev())
+        self.dist.all_reduce(t, op=self.dist.ReduceOp.MIN, group=self.group)
+        return int(t.item())
+
+    def gather0(self, X, gid):
+        """All points (X, gid) to rank 0, ordered by gid (None on the other ranks)."""
+        torch = self.torch
+        xs = self._all_gather_1d(X.reshape(-1).float())
+        gs = self._all_gather_1d(gid.long())
+        if self.rank != 0:
+            return None
+        order = torch.argsort(gs)
+        return xs.reshape(-1, self.d)[order.to(xs.device)], gs[order]
+
+
+def run_sharded(X_own, gid_own, eps: float, ex: ShardExchange, make_ctx, max_iters: int = 10000):
+    """Algorithm 4 (L258-278) over sharded points.
+
+    X_own   : (n_r, d) float32 tensor, this rank's initial share of the points
+    gid_own : (n_r,) int64 tensor, their global indices (0..n-1)
+    make_ctx: callable(n_local, d) -> a context (eggsync.Context or a stand-in) for own + halo
+    Returns (iters, converged, labels, coords) on rank 0 (labels / coords in global index
+    order), (iters, converged, None, None) elsewhere.
+    """
+    torch = ex.torch
+    d = ex.d
+    X, gid = X_own, gid_own
+    t, synced = 0, False
+    verified = None
+    while True:
+        split = ex.splitters(X[:, 0])
+        Xo, go, Xh, gh = ex.exchange(X, gid, split)
+        n_own = Xo.shape[0]
+        ctx = make_ctx(n_own + Xh.shape[0], d)
+        loc = torch.cat([Xo, Xh]).contiguous()
+        ctx.load(loc.cpu().numpy() if not loc.is_cuda else loc)
+        ctx.set_own(n_own)
+        ctx.build()
+        ctx.update()
+        f1 = ex.min(ctx.flags()[0])                        # first term over all own points
+        f2 = -1
+        if f1 == 1:
+            ctx.second_term()
+            f2 = ex.min(ctx.flags()[1])
+        synced = f1 == 1 and f2 == 1
+        ctx.advance()
+        nxt = ctx.coords()
+        nxt = torch.as_tensor(nxt, device=X.device)[:n_own]
+        if synced:
+            verified = (Xo, go)                            # D^t: its cells are the clusters (R7)
+        X, gid = nxt, go
+        t += 1
+        if hasattr(ctx, "close"):
+            ctx.close()
+        if synced or t >= max_iters:
+            break
+    final = ex.gather0(X, gid)
+    state = ex.gather0(*(verified if synced else (X, gid)))
+    if ex.rank != 0:
+        return t, synced, None, None
+    Xs = state[0].contiguous()
+    ctx = make_ctx(Xs.shape[0], d)
+    ctx.load(Xs.cpu().numpy() if not Xs.is_cuda else Xs)
+    ctx.build()
+    labels = ctx.labels()                                  # cells of the verified state (L256)
+    if hasattr(ctx, "close"):
+        ctx.close()
+    return t, synced, labels, final[0]

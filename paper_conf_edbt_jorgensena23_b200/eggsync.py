@@ -27,7 +27,7 @@ SYMBOLS = [
     "eggsync_ctx_unpack", "eggsync_ctx_advance", "eggsync_ctx_labels", "eggsync_ctx_coords",
     "eggsync_ctx_run", "eggsync_ctx_stream", "eggsync_ctx_work", "eggsync_ctx_tc_work", "eggsync_ctx_launches",
     "eggsync_release_cache", "eggsync_ctx_update_owned", "eggsync_ctx_owned_count", "eggsync_ctx_pack_owned",
-    "eggsync_ctx_unpack_owned", "eggsync_ctx_plan_owned", "eggsync_ctx_update_planned", "eggsync_sync_step",
+    "eggsync_ctx_unpack_owned", "eggsync_ctx_plan_owned", "eggsync_ctx_update_planned", "eggsync_ctx_set_own", "eggsync_sync_step",
     "eggsync_sync_lambda",
 ]
 
@@ -102,6 +102,7 @@ def lib():
             "eggsync_ctx_unpack_owned": ([vp, vp, i32], ctypes.c_int),
             "eggsync_ctx_plan_owned": ([vp, i32, i32, vp], ctypes.c_int),
             "eggsync_ctx_update_planned": ([vp, i32, i32, vp], ctypes.c_int),
+            "eggsync_ctx_set_own": ([vp, i64], ctypes.c_int),
             "eggsync_sync_step": ([vp, i64, i32, f32, i32, vp, vp], ctypes.c_int),
             "eggsync_sync_lambda": ([vp, i64, i32, f32, ctypes.c_double, i32, i32, vp, vp], ctypes.c_int),
         }
@@ -354,6 +355,10 @@ class Context:
 
     def pack_owned_into(self, rank: int, ranks: int, tensor):
         _check(lib().eggsync_ctx_pack_owned(self.h, rank, ranks, ctypes.c_void_p(tensor.data_ptr())))
+
+    def set_own(self, n_own: int):
+        """Sharded runs: the first n_own loaded points are this rank's own (criterion flags)."""
+        _check(lib().eggsync_ctx_set_own(self.h, n_own))
 
     def plan_owned(self, rank: int, ranks: int):
         """Plan pass of the owned tiles; returns int64[6] statistics (see eggsync.h)."""
