@@ -274,6 +274,7 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st, do
       {(void**)&c_minorig, sizeof(uint32_t) * cap},
       {(void**)&nbr, sizeof(int32_t) * n},
       {(void**)&lab_final, sizeof(int32_t) * n},
+      {(void**)&second_need, sizeof(uint8_t) * cap},
       {(void**)&work, sizeof(unsigned long long) * 8},
       {(void**)&co_of, sizeof(int32_t) * n},
       {(void**)&full_S, d <= 16 ? sizeof(double) * 2 * d * n : 0},

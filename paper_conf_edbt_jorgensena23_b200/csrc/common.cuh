@@ -229,6 +229,7 @@ struct Workspace {
   uint32_t* c_minorig = nullptr;
   int32_t* nbr = nullptr;      // optional neighbour counts (sorted order)
   int32_t* lab_final = nullptr; // labels recorded when the criterion held (original order)
+  uint8_t* second_need = nullptr;  // [cap] grid cells whose points need the second term's point test
   bool have_final = false;
   bool second_checked = false;
   int64_t bytes = 0;

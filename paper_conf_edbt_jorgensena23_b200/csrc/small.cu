@@ -76,6 +76,7 @@ __global__ void __launch_bounds__(kSmThreads, 1) k_cluster_small(const SmallArgs
   const int tid = threadIdx.x;
 
   for (int k = tid; k < n * D; k += kSmThreads) xb[0][k] = a.x0[k];
+  __syncthreads();  // D^0 complete before the first keys read it (racecheck)
   const int per = (n + kSmCtas - 1) / kSmCtas;  // own points [rank*per, rank*per + per)
   const int p0 = rank * per, p1 = min(n, p0 + per);
   int cur = 0, t = 0;

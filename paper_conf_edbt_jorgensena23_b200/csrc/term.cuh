@@ -32,6 +32,8 @@ struct TermArgs {
   float e2f, ed2f, edf, rel;
   double e2d, ed2d;
   int32_t* flags;  // [1] second term AND, [3] error
+  const uint8_t* __restrict__ need;  // per grid cell: its points need the point-level test (nullptr: all)
+  int32_t n_grid;
 };
 
 // dist(MBR, p)^2 exactly as the oracle evaluates it (L110; fp64, dimension order)
@@ -56,7 +58,8 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_second(const TermArgs<D> 
   const int wid = threadIdx.x >> 5, lane = threadIdx.x & 31;
   int2* stk = reinterpret_cast<int2*>(smem) + wid * a.stack_len;
   const int64_t j = a.lo + ((int64_t)blockIdx.x * kWarpsPerCta + wid) * 32 + lane;
-  const bool valid = j < a.hi && (!a.orig || a.orig[j] < (uint32_t)a.n_own);  // halo points do not test
+  bool valid = j < a.hi && (!a.orig || a.orig[j] < (uint32_t)a.n_own);  // halo points do not test
+  if (valid && a.need) valid = a.need[a.g_of[j]] != 0;  // cells cleared by the cell-level pass
   const unsigned amask = __ballot_sync(FULLMASK, valid);
   if (amask == 0u) return;
   float p[D];
@@ -177,6 +180,86 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32) k_second(const TermArgs<D> 
   if (__any_sync(FULLMASK, viol) && lane == 0) atomicAnd(&a.flags[1], 0);
 }
 
+// Cell-level pre-pass of the second term (one thread per grid cell A, its MBR standing for
+// its points): a unit u of another cell B can host a violating pair (p in A, q in u) only if
+//   MINDIST(MBR_u, MBR_A) <= eps + delta  (some pair within eps + delta),
+//   MINDIST(MBR_B, MBR_A) <= eps          (some p of A with dist(MBR_B, p) <= eps, L108-110), and
+//   MAXDIST(MBR_u, MBR_A) >  eps          (some pair beyond eps: a shell pair is possible),
+// all tested in fp32 with the rel margins (conservative: an undecided case needs the point test).
+// Cells for which no unit passes need no point-level test; near convergence that is almost all
+// of them (collapsed clusters are single cells), so the point pass runs on a few points only.
+template <int D>
+__global__ void __launch_bounds__(128) k_second_cells(const TermArgs<D> a, int32_t ng, const int32_t* __restrict__ u2co,
+                                                      uint8_t* __restrict__ need) {
+  constexpr int BS = ceil4(2 * D);
+  const int32_t A = (int32_t)((int64_t)blockIdx.x * blockDim.x + threadIdx.x);
+  if (A >= ng) return;
+  float lo[D], hi[D];
+#pragma unroll
+  for (int i = 0; i < D; ++i) {
+    lo[i] = ordf(a.g_lo[(int64_t)i * a.cap + A]);
+    hi[i] = ordf(a.g_hi[(int64_t)i * a.cap + A]);
+  }
+  const float lim_ed = a.ed2f * (1.f + a.rel), e_out = a.e2f * (1.f + a.rel), e_in = a.e2f * (1.f - a.rel);
+  // box-box distances: min over the boxes' gap, max over their farthest corners
+  auto mind_box = [&](const float* bl, const float* bh) {
+    float m = 0.f;
+#pragma unroll
+    for (int i = 0; i < D; ++i) {
+      const float g = fmaxf(fmaxf(bl[i] - hi[i], lo[i] - bh[i]), 0.f);
+      m = fmaf(g, g, m);
+    }
+    return m;
+  };
+  int stk[96];
+  int sp = 0;
+  stk[sp++] = a.nc > 1 ? 0 : (int)kLeafBit;
+  bool needed = false;
+  while (sp > 0 && !needed) {
+    const int node = stk[--sp];
+    if (node & (int)kLeafBit) {
+      const int32_t u = node & 0x7fffffff;
+      const int32_t B = u2co ? u2co[u] : u;
+      if (B == A) continue;
+      float ul[D], uh[D], bl[D], bh[D];
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        ul[i] = ordf(a.c_lo[(int64_t)i * a.cap + u]);
+        uh[i] = ordf(a.c_hi[(int64_t)i * a.cap + u]);
+        bl[i] = ordf(a.g_lo[(int64_t)i * a.cap + B]);
+        bh[i] = ordf(a.g_hi[(int64_t)i * a.cap + B]);
+      }
+      if (mind_box(ul, uh) > lim_ed) continue;
+      if (mind_box(bl, bh) > e_out) continue;
+      float mx = 0.f;
+#pragma unroll
+      for (int i = 0; i < D; ++i) {
+        const float g = fmaxf(uh[i] - lo[i], hi[i] - ul[i]);
+        mx = fmaf(g, g, mx);
+      }
+      if (mx <= e_in) continue;
+      needed = true;
+      continue;
+    }
+    const float* __restrict__ bx = a.t_box + (int64_t)node * BS;
+    float bl[D], bh[D];
+#pragma unroll
+    for (int i = 0; i < D; ++i) {
+      bl[i] = bx[i];
+      bh[i] = bx[D + i];
+    }
+    if (mind_box(bl, bh) > lim_ed) continue;
+    if (sp + 2 > 96) {
+      needed = true;  // too deep for the private stack: leave it to the point pass
+      break;
+    }
+    const int4 meta = a.t_meta[node];
+    stk[sp++] = meta.w;
+    stk[sp++] = meta.z;
+  }
+  need[A] = needed ? 1 : 0;
+}
+
 template <int D>
 int run_second_term(Workspace& ws, int64_t lo, int64_t hi) {
   if (hi <= lo) return EGGSYNC_OK;
@@ -209,6 +292,15 @@ int run_second_term(Workspace& ws, int64_t lo, int64_t hi) {
   a.e2d = ws.k.e2;
   a.ed2d = ws.k.ed2;
   a.flags = ws.flags;
+  a.need = nullptr;
+  a.n_grid = ws.n_grid;
+  if (ws.n_grid >= 2 && ws.second_need) {  // cell-level pass first: which cells need the point test
+    k_second_cells<D><<<(unsigned)((ws.n_grid + 127) / 128), 128, 0, ws.stream>>>(a, ws.n_grid, ws.g_u2co,
+                                                                                ws.second_need);
+    ws.launches += 1;
+    EGG_CUDA(cudaGetLastError());
+    a.need = ws.second_need;
+  }
   const size_t smem = (size_t)kWarpsPerCta * a.stack_len * sizeof(int2);
   EGG_CUDA(cudaFuncSetAttribute(k_second<D>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   const int64_t per = 32 * kWarpsPerCta;

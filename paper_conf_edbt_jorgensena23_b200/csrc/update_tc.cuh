@@ -125,7 +125,7 @@ __device__ __forceinline__ int64_t tc_tile_base(int64_t lo, int64_t tile, int32_
 }
 
 template <int D>
-__global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a) {
+__global__ void __launch_bounds__(kPlanWarps * 32, 3) k_tc_plan(const PlanArgs<D> a) {
   constexpr int kP = 4;
   constexpr int BS = ceil4(2 * D);
   extern __shared__ __align__(16) unsigned char psm[];
@@ -282,15 +282,28 @@ __global__ void __launch_bounds__(kPlanWarps * 32) k_tc_plan(const PlanArgs<D> a
 #pragma unroll
         for (int k = 0; k < kP; ++k) anyf |= fm[k] != 0u;
         if (anyf) {
-          const float* __restrict__ sm = a.t_sum + (int64_t)node * BS;
+          const float4* __restrict__ sm4 = reinterpret_cast<const float4*>(a.t_sum + (int64_t)node * BS);
+          float sm[BS];
+#pragma unroll
+          for (int k = 0; k < BS / 4; ++k) {
+            const float4 t4 = sm4[k];
+            sm[4 * k] = t4.x;
+            sm[4 * k + 1] = t4.y;
+            sm[4 * k + 2] = t4.z;
+            sm[4 * k + 3] = t4.w;
+          }
 #pragma unroll
           for (int k = 0; k < kP; ++k) {
             if (full[k]) {
               N[k] += tcn[b];
+              // loads before stores, D at a time: the read-modify-writes overlap (two latencies)
 #pragma unroll
-              for (int i = 0; i < 2 * D; ++i) {
-                double* dst = a.full_S + (int64_t)i * a.n + j[k];
-                *dst = (touched[k] ? *dst : 0.0) + (double)sm[i];
+              for (int h = 0; h < 2; ++h) {
+                double cur[D];
+#pragma unroll
+                for (int i = 0; i < D; ++i) cur[i] = touched[k] ? a.full_S[(int64_t)(h * D + i) * a.n + j[k]] : 0.0;
+#pragma unroll
+                for (int i = 0; i < D; ++i) a.full_S[(int64_t)(h * D + i) * a.n + j[k]] = cur[i] + (double)sm[h * D + i];
               }
               touched[k] = true;
             }
@@ -527,7 +540,7 @@ __device__ __forceinline__ void tc_rare(const TcArgs<D>& a, const float* __restr
 // Build entry slot `pt` (unit c, or padding when c < 0) of a stage: B1 row and metadata from
 // the unit's record head (prefetched into registers); its digit row (B2) came by cp.async.
 template <int D>
-__device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const TcMisc* __restrict__ ms,
+__device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const float (&o)[D],
                                                 const TcStage<D>& st, int pt, int32_t c,
                                                 const float* __restrict__ rec, float Rq, float Rqi) {
   using C = TcCfg<D>;
@@ -545,26 +558,33 @@ __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const TcMisc
       r[4 * k + 2] = t4.z;
       r[4 * k + 3] = t4.w;
     }
-    float cc = 0.f, cinf = 0.f;
+    float cc0 = 0.f, cc1 = 0.f, cinf = 0.f;  // two independent chains (latency)
 #pragma unroll
     for (int i = 0; i < D; ++i) {
-      const float cp = r[i] - ms->o[i];
+      const float cp = r[i] - o[i];
       const float h = tc::tf32_hi(cp);
       b[i] = -2.f * h;
       b[D + i] = -2.f * h;
       b[2 * D + i] = -2.f * (cp - h);
-      cc = fmaf(cp, cp, cc);
+      if (i & 1) cc1 = fmaf(cp, cp, cc1);
+      else cc0 = fmaf(cp, cp, cc0);
       cinf = fmaxf(cinf, fabsf(cp));
     }
+    const float cc = cc0 + cc1;
     const float rad = r[D];
-    // error budget: eta = rounding of the shifted frame; E = tf32 split
-    // (2^-17 |q||c'|) + tensor-core accumulation (4 K-steps x 9 terms x 2^-23 of the sum
-    // of |terms| <= 2^-17.8 (2|q||c'| + |L|)) + fp32 |q|^2, |c'|^2, L and v roundings
+    // error budget: eta = rounding of the shifted frame; E bounds |v - v_exact|:
+    //   tf32 split of -2 q.c' (3 products; lo parts truncated to tf32, lo*lo dropped):
+    //     <= 2 * 3 * 2^-20 sum|q_i||c'_i| <= 2^-17.4 |q||c'|               (Cauchy-Schwarz)
+    //   tensor-core accumulation, 4 K-steps of 8 products + accumulator, each truncating
+    //     <= 9 * 2^-23 of the sum of |terms| (2|q||c'| + |L|):  <= 2^-16.8 |q||c'| + 2^-17.8 |L|
+    //   L = limF - |c'|^2 split hi/lo (2^-20 |L|); fp32 |q|^2, |c'|^2 (D FMAs): (D+2) u (|q|^2 + cc)
+    //   => E <= 2^-16 Rq|c'| + 2^-17 |L| + 2^-20 (Rq^2 + cc)   (Rq >= |q|, D <= 12)
     const float eta = 2.5f * kU * sqrtf((float)D) * (Rqi + cinf);
     const float ep = (a.e + rad) * (1.f + 8.f * kU) + eta;
     const float em = (a.e - rad) * (1.f - 8.f * kU) - eta;
     const float limF0 = em > 0.f ? em * em * (1.f - 4.f * kU) : -1.f;
-    const float E = 1.52587890625e-05f * (2.f * Rq * sqrtf(cc) + fabsf(limF0 - cc) + cc + Rq * Rq + 1e-30f);
+    const float E = 1.52587890625e-05f * (Rq * sqrtf(cc)) + 7.62939453125e-06f * fabsf(limF0 - cc) +
+                    9.5367431640625e-07f * (cc + Rq * Rq) + 1e-30f;
     const float limF = em > 0.f ? limF0 - E : -1.f;
     const float limO = ep * ep * (1.f + 4.f * kU) + E;
     W = (limO - limF) * (1.f + 4.f * kU);
@@ -758,6 +778,9 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
     const int pt = tid - 256;  // entry slot 0..127
     const int pw = pt >> 5;
     const float Rq = ms->Rq, Rqi = ms->Rqi;
+    float ov[D];  // tile origin, in registers for the operand builds
+#pragma unroll
+    for (int i = 0; i < D; ++i) ov[i] = ms->o[i];
     const int nchunk = N2 / 16;
     const int32_t* __restrict__ ent = a.ent + a.eoff[tile];
     // copies of entry tile t into its stage (one cp.async group per tile, empty beyond T)
@@ -819,7 +842,7 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
       TCP_T(p2);
       TCP_ADD(1, p2 - p1);
       TcStage<D> st(ring, bp.i, SB, N2);
-      const float W = tc_build_entry<D>(a, ms, st, pt, st.cell[pt], st.rec + pt * C::R0S, Rq, Rqi);
+      const float W = tc_build_entry<D>(a, ov, st, pt, st.cell[pt], st.rec + pt * C::R0S, Rq, Rqi);
       // chunk maximum of the band widths (W >= 0: its bits order as unsigned integers)
       const uint32_t wm = __reduce_max_sync(FULLMASK, __float_as_uint(W));
       if (lane == 0) st.wmax[pw] = __uint_as_float(wm);
