@@ -1222,8 +1222,14 @@ int run_planned_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr, int64_t 
                                                                     ws.tc_eoff, ws.tc_ent, (int32_t)owned);
     EGG_CUDA(cudaGetLastError());
     ws.launches += 1;
-    // launch order: point tiles by descending entry count (longest-processing-time first)
-    {
+    // launch order: point tiles by descending entry count (longest-processing-time first);
+    // EGGSYNC_TC_ORDER=0: the sorted (spatial) order, better L2 reuse of neighbouring tiles' cells
+    static const int order_env = [] {
+      const char* e = getenv("EGGSYNC_TC_ORDER");
+      return e ? atoi(e) : 1;
+    }();
+    const bool heavy_first = order_env != 0;
+    if (heavy_first) {
       size_t stmp = 0;
       EGG_CUDA(cub::DeviceRadixSort::SortPairsDescending(nullptr, stmp, ws.tc_ne, ws.tc_pk, ws.tc_pv, ws.tc_perm,
                                                          (int)owned, 0, 32, ws.stream));
@@ -1269,7 +1275,7 @@ int run_planned_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr, int64_t 
     a.c_hi = ws.c_hi;
     a.ent = ws.tc_ent;
     a.eoff = ws.tc_eoff;
-    a.perm = ws.tc_perm;
+    a.perm = heavy_first ? ws.tc_perm : ws.tc_pv;
     a.t_ne = ws.tc_ne;
     a.full_S = ws.full_S;
     a.full_N = ws.full_N;
