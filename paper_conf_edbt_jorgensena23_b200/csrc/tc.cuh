@@ -5,6 +5,8 @@
 // ISA (the same fields CuTe's UMMA::SmemDescriptor / UMMA::InstrDescriptor
 // name).  Product path only; nothing here is shared with oracle/.
 #pragma once
+#include <cuda_fp16.h>
+
 #include <cstdint>
 
 namespace egg {
@@ -87,6 +89,32 @@ __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t
 __host__ __device__ constexpr uint32_t idesc_tf32(int M, int N, bool b_mn_major) {
   return (1u << 4) | (2u << 7) | (2u << 10) | ((b_mn_major ? 1u : 0u) << 16) | ((uint32_t)(N >> 3) << 17) |
          ((uint32_t)(M >> 4) << 24);
+}
+
+// ---- instruction descriptor: kind::f16, fp16 A and B (K-major), fp32 accumulate ----
+//  bits [4,6) D format (1 = F32), [7,10) A format (0 = F16), [10,13) B format (0 = F16)
+__host__ __device__ constexpr uint32_t idesc_f16(int M, int N) {
+  return (1u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
+}
+// D[tmem] (+)= A[tmem] * B[smem]^T, fp16 x fp16 -> fp32 (A: M x 16 fp16 = 8 TMEM columns)
+__device__ __forceinline__ void mma_ts_f16(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
+                                           uint32_t accumulate) {
+  asm volatile(
+      "{\n .reg .pred p;\n setp.ne.b32 p, %4, 0;\n"
+      " tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n}" ::"r"(d_tmem),
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+// two fp32 values as a packed fp16 pair (round to nearest; x in the low half)
+__device__ __forceinline__ uint32_t pack_h2(float x, float y) {
+  uint32_t r;
+  asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(r) : "f"(y), "f"(x));
+  return r;
+}
+// fp16 hi / lo split of x (|x| << 65504): hi = fp16(x), lo = fp16(x - hi)
+__device__ __forceinline__ void split_h(float x, float& hi, float& lo) {
+  hi = __half2float(__float2half_rn(x));
+  lo = __half2float(__float2half_rn(x - hi));
 }
 
 // ---- instruction descriptor: kind::i8, signed 8-bit A and B, s32 accumulate ----

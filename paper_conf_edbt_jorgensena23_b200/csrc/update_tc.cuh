@@ -60,7 +60,8 @@ constexpr int kTcMaxStages = 8;
 
 template <int D>
 struct TcCfg {
-  static constexpr int K1 = ((3 * D + 2) + 7) / 8 * 8;  // GEMM1 K: q_hi, q_lo, q_hi, 1, 1
+  static constexpr int K1 = ((3 * D + 2) + 15) / 16 * 16;  // GEMM1 K (fp16): q_hi, q_lo, q_hi, s, s
+  static constexpr int QC = K1 / 2;                        // TMEM columns of Q (two fp16 per column)
   static constexpr int NV = 2 * D + 1;                  // sin, cos, count
   static constexpr int DB = CellDig<D>::kBytes;         // digit row of a cell (GEMM2 N <= DB)
   static constexpr int R = CellRec<D>::kFloats;
@@ -68,8 +69,8 @@ struct TcCfg {
   static constexpr int R0S = (R0 / 4) % 2 == 0 ? R0 + 4 : R0;  // shared stride: conflict-free 16-B accesses
   static constexpr int kRecBytes = kTcEnt * R0S * 4;   // record heads of a stage's entries (cp.async)
   // shared memory: ring stages (run-time size, TcStage) | raw record heads | rare sums | misc
-  static constexpr int SBO1 = (K1 / 4) * 128;
-  static constexpr int kB1Bytes = kTcEnt * K1 * 4;
+  static constexpr int SBO1 = (K1 / 8) * 128;
+  static constexpr int kB1Bytes = kTcEnt * K1 * 2;
   static constexpr int kRareBytes = NV * kTcTile * 8;   // exact sums [2D][row] (2^-32) + count [row]
   static constexpr int kSlotBytes = 4 * kTcEnt * 4;     // slot units of 4 entry tiles (producers' ring)
   static constexpr int kMiscBytes = 1024;
@@ -454,7 +455,7 @@ __device__ __forceinline__ void cp_async_wait() {
 }
 
 // One ring stage (run-time size: GEMM2 N = n2 depends on the digits needed):
-//   b1   [kTcEnt][K1] tf32, K-major core matrices (GEMM1 B: entry rows)            (producers)
+//   b1   [kTcEnt][K1] fp16, K-major core matrices (GEMM1 B: entry rows)            (producers)
 //   b2   [n2/16][kTcEnt][16] int8, MN-major core matrices (GEMM2 B: digits x entries) (cp.async)
 //   rec  [kTcEnt][R0S] record heads: centre (= the point of a singleton), radius, count, start (cp.async)
 //   W, cell [kTcEnt] band width and unit of every slot (-1 = padding); wmax[4]       (producers)
@@ -539,6 +540,11 @@ __device__ __forceinline__ void tc_rare(const TcArgs<D>& a, const float* __restr
 
 // Build entry slot `pt` (unit c, or padding when c < 0) of a stage: B1 row and metadata from
 // the unit's record head (prefetched into registers); its digit row (B2) came by cp.async.
+// GEMM1 runs in fp16 on values scaled by kTcScale = 2^8 (the products and v by 2^16): shifted
+// coordinates |c'|, |q'| <= 1 become <= 256 (fp16 max 65504), their low halves stay normal.
+constexpr float kTcScale = 256.f;
+constexpr float kTcScale2 = 65536.f;
+
 template <int D>
 __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const float (&o)[D],
                                                 const TcStage<D>& st, int pt, int32_t c,
@@ -562,10 +568,11 @@ __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const float 
 #pragma unroll
     for (int i = 0; i < D; ++i) {
       const float cp = r[i] - o[i];
-      const float h = tc::tf32_hi(cp);
+      float h, l;
+      tc::split_h(cp * kTcScale, h, l);
       b[i] = -2.f * h;
       b[D + i] = -2.f * h;
-      b[2 * D + i] = -2.f * (cp - h);
+      b[2 * D + i] = -2.f * l;
       if (i & 1) cc1 = fmaf(cp, cp, cc1);
       else cc0 = fmaf(cp, cp, cc0);
       cinf = fmaxf(cinf, fabsf(cp));
@@ -573,12 +580,12 @@ __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const float 
     const float cc = cc0 + cc1;
     const float rad = r[D];
     // error budget: eta = rounding of the shifted frame; E bounds |v - v_exact|:
-    //   tf32 split of -2 q.c' (3 products; lo parts truncated to tf32, lo*lo dropped):
-    //     <= 2 * 3 * 2^-20 sum|q_i||c'_i| <= 2^-17.4 |q||c'|               (Cauchy-Schwarz)
-    //   tensor-core accumulation, 4 K-steps of 8 products + accumulator, each truncating
-    //     <= 9 * 2^-23 of the sum of |terms| (2|q||c'| + |L|):  <= 2^-16.8 |q||c'| + 2^-17.8 |L|
-    //   L = limF - |c'|^2 split hi/lo (2^-20 |L|); fp32 |q|^2, |c'|^2 (D FMAs): (D+2) u (|q|^2 + cc)
-    //   => E <= 2^-16 Rq|c'| + 2^-17 |L| + 2^-20 (Rq^2 + cc)   (Rq >= |q|, D <= 12)
+    //   fp16 split of -2 q.c' (round-to-nearest hi, lo rounded again, lo*lo dropped):
+    //     <= 2 * 3 * 2^-22 sum|q_i||c'_i| <= 2^-19.4 |q||c'|               (Cauchy-Schwarz)
+    //   tensor-core accumulation, 2 K-steps of 16 products + accumulator, each truncating
+    //     <= 17 * 2^-23 of the sum of |terms| (2|q||c'| + |L|):  <= 2^-16.9 |q||c'| + 2^-17.9 |L|
+    //   L = limF - |c'|^2 split hi/lo (2^-22 |L|); fp32 |q|^2, |c'|^2 (D FMAs): (D+2) u (|q|^2 + cc)
+    //   => E <= 2^-16 Rq|c'| + 2^-17 |L| + 2^-20 (Rq^2 + cc)   (Rq >= |q|, D <= 12); unscaled
     const float eta = 2.5f * kU * sqrtf((float)D) * (Rqi + cinf);
     const float ep = (a.e + rad) * (1.f + 8.f * kU) + eta;
     const float em = (a.e - rad) * (1.f - 8.f * kU) - eta;
@@ -587,24 +594,27 @@ __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const float 
                     9.5367431640625e-07f * (cc + Rq * Rq) + 1e-30f;
     const float limF = em > 0.f ? limF0 - E : -1.f;
     const float limO = ep * ep * (1.f + 4.f * kU) + E;
-    W = (limO - limF) * (1.f + 4.f * kU);
+    W = (limO - limF) * (1.f + 4.f * kU) * kTcScale2;  // in the scaled units of v
     const float L = limF - cc;
-    const float Lh = tc::tf32_hi(L);
+    float Lh, Ll;
+    tc::split_h(L * kTcScale, Lh, Ll);  // times A's s = 2^8 column: L * 2^16
     b[3 * D] = -Lh;
-    b[3 * D + 1] = -(L - Lh);
+    b[3 * D + 1] = -Ll;
   } else {
 #pragma unroll
     for (int k = 0; k < 3 * D + 2; ++k) b[k] = 0.f;
-    b[3 * D] = 1073741824.f;  // v = 2^30: outside, never ambiguous
+    b[3 * D] = 60000.f;  // v = 2^8 * 60000: far outside, never ambiguous
   }
 #pragma unroll
   for (int k = 3 * D + 2; k < K1; ++k) b[k] = 0.f;
-  // B1: K-major, entry rows
+  // B1: K-major fp16, entry rows (8 K-values per 16-byte core-matrix row)
   {
     unsigned char* b1 = reinterpret_cast<unsigned char*>(st.b1) + (pt >> 3) * C::SBO1 + (pt & 7) * 16;
 #pragma unroll
-    for (int kc = 0; kc < K1 / 4; ++kc)
-      *reinterpret_cast<float4*>(b1 + kc * 128) = make_float4(b[4 * kc], b[4 * kc + 1], b[4 * kc + 2], b[4 * kc + 3]);
+    for (int kc = 0; kc < K1 / 8; ++kc)
+      *reinterpret_cast<uint4*>(b1 + kc * 128) =
+          make_uint4(tc::pack_h2(b[8 * kc], b[8 * kc + 1]), tc::pack_h2(b[8 * kc + 2], b[8 * kc + 3]),
+                     tc::pack_h2(b[8 * kc + 4], b[8 * kc + 5]), tc::pack_h2(b[8 * kc + 6], b[8 * kc + 7]));
   }
   st.W[pt] = W;
   return W;
@@ -662,7 +672,7 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
   const int64_t base = tc_tile_base(a.lo, tile, a.stride, a.offset);
   const int32_t ne = a.t_ne[tile];
   const int T = (ne + kTcEnt - 1) / kTcEnt;  // entry tiles (the slot list is padded to T * kTcEnt)
-  const int kColS = K1, kColO = K1 + NS * kTcEnt;
+  const int kColS = C::QC, kColO = C::QC + NS * kTcEnt;
 #ifdef EGG_TC_PROF
   unsigned long long prof_acc[4] = {0, 0, 0, 0};
 #endif
@@ -729,7 +739,7 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
       s = fmaf(q[i], q[i], s);
       rinf = fmaxf(rinf, fabsf(q[i]));
     }
-    if (valid) pp = s;
+    if (valid) pp = s * kTcScale2;  // v is formed in the scaled units of GEMM1
     if (grp == 0) {
       float r2 = sqrtf(s) * (1.f + 4.f * kU), ri = rinf;
 #pragma unroll
@@ -741,25 +751,26 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
         atomicMax(reinterpret_cast<int*>(&ms->Rq), __float_as_int(r2));
         atomicMax(reinterpret_cast<int*>(&ms->Rqi), __float_as_int(ri));
       }
-      // Q row -> TMEM columns [0, K1): q_hi, q_lo, q_hi, 1, 1, 0...
-      uint32_t v[K1];
+      // Q row -> TMEM columns [0, K1/2) as fp16 pairs (scaled by 2^8): q_hi, q_lo, q_hi, s, s, 0...
+      float v[K1];
 #pragma unroll
       for (int i = 0; i < D; ++i) {
-        const float h = tc::tf32_hi(q[i]);
-        v[i] = __float_as_uint(h);
-        v[D + i] = __float_as_uint(q[i] - h);
-        v[2 * D + i] = __float_as_uint(h);
+        float h, l;
+        tc::split_h(q[i] * kTcScale, h, l);
+        v[i] = h;
+        v[D + i] = l;
+        v[2 * D + i] = h;
       }
-      v[3 * D] = __float_as_uint(1.f);
-      v[3 * D + 1] = __float_as_uint(1.f);
+      v[3 * D] = kTcScale;
+      v[3 * D + 1] = kTcScale;
 #pragma unroll
-      for (int k = 3 * D + 2; k < K1; ++k) v[k] = 0u;
+      for (int k = 3 * D + 2; k < K1; ++k) v[k] = 0.f;
       const uint32_t taddr = ms->tbase + ((uint32_t)(32 * (wid & 3)) << 16);
 #pragma unroll
-      for (int c = 0; c < K1 / 8; ++c) {
+      for (int c = 0; c < K1 / 16; ++c) {
         uint32_t w8[8];
 #pragma unroll
-        for (int k = 0; k < 8; ++k) w8[k] = v[8 * c + k];
+        for (int k = 0; k < 8; ++k) w8[k] = tc::pack_h2(v[16 * c + 2 * k], v[16 * c + 2 * k + 1]);
         tc::st8(taddr + 8 * c, w8);
       }
       tc::wait_st();
@@ -857,7 +868,7 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
   if (wid == kMma1Warp && lane == 0) {
     // ================================ GEMM1 issue ================================
     // S[jt % NS] = Q . B1(jt)^T once stage jt is built and GEMM2(jt - NS) released the buffer.
-    constexpr uint32_t id1 = tc::idesc_tf32(128, kTcEnt, false);
+    constexpr uint32_t id1 = tc::idesc_f16(128, kTcEnt);
     const uint32_t ring_s = tc::smem_addr(ring);
     RingPos sp, bq;
     for (int jt = 0; jt < T; ++jt) {
@@ -872,8 +883,8 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
       tc::fence_after();
       const uint32_t b1 = ring_s + s * SB;
 #pragma unroll
-      for (int k = 0; k < K1 / 8; ++k)
-        tc::mma_ts(tb + kColS + kTcEnt * b, tb + 8 * k, tc::sdesc(b1 + k * 256, 128, C::SBO1), id1, k > 0);
+      for (int k = 0; k < K1 / 16; ++k)  // 16 fp16 K-values per MMA: 8 TMEM columns of A, 2 core matrices of B
+        tc::mma_ts_f16(tb + kColS + kTcEnt * b, tb + 8 * k, tc::sdesc(b1 + k * 256, 128, C::SBO1), id1, k > 0);
       tc::mma_commit(&ms->s_full[b]);
       sp.adv(NST);
       bq.adv(NS);
@@ -1248,11 +1259,11 @@ int run_planned_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr, int64_t 
     int ndig = 3;
     while (ndig < kDigMax && (double)maxc * (double)(1 << kDigF) + 1.0 > 0.498 * std::ldexp(1.0, 8 * ndig)) ++ndig;
     const int n2 = (ndig * C::NV + 15) / 16 * 16;
-    const int ns = (C::K1 + 3 * kTcEnt + n2 <= 512) ? 3 : 2;  // S buffers that fit TMEM next to Q and O
+    const int ns = (C::QC + 3 * kTcEnt + n2 <= 512) ? 3 : 2;  // S buffers that fit TMEM next to Q and O
     const int sbytes = C::stage_bytes(n2);
     int nst = (C::kBudget - C::kFixedBytes) / sbytes;
     nst = nst > kTcMaxStages ? kTcMaxStages : nst;
-    if (nst < 2 || C::K1 + 2 * kTcEnt + n2 > 512) {  // cannot happen for D <= kTcMaxD
+    if (nst < 2 || C::QC + 2 * kTcEnt + n2 > 512) {  // cannot happen for D <= kTcMaxD
       ws.tc_used = 0;
       return run_update_simt<D>(ws, lo, hi, nbr);
     }
