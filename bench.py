@@ -242,31 +242,42 @@ def run_ours(args):
     fmax = (peaks or {}).get("sm_max_mhz") or clk_s["sm_max_mhz"] or 1965.0
     upd_share = sum(upd_ms) / sum(step_ms)
     if tcw["launches"] > 0:
-        # roofline of the dominant kernel, k_update_tc: tf32 tensor cores.  achieved = the
+        # roofline of the dominant kernel, k_update_tc: tcgen05 tensor cores.  achieved = the
         # METHOD's FLOPs per launch / the kernel's own event time (CUDA events on the library
         # stream, every launch of the timed region).  Method FLOPs per (point, entry) pair
-        # (DESIGN.md §6): the expanded distance |p-c|^2 - lim = -2 q.c' - L, d+2 MACs, plus the
-        # masked Eq.5 sums P.[sum sin | sum cos | count], 2d+1 MACs: 2((d+2)+(2d+1)) FLOPs.
-        # The hi/lo tf32 splits that make those products ~fp32-exact are emulation overhead,
-        # reported separately (emulated_flops_per_step), not counted as achieved work.
+        # (DESIGN.md §6): the expanded distance |p-c|^2 - lim = -2 q.c' - L, d+2 MACs (GEMM1,
+        # kind::f16), plus the masked Eq.5 sums P.[sum sin | sum cos | count], 2d+1 MACs (GEMM2,
+        # kind::i8): 2((d+2)+(2d+1)) FLOPs.  The hi/lo fp16 splits and base-256 digit columns
+        # that make those products exact are emulation overhead, reported separately
+        # (emulated_flops_per_step), not counted as achieved work.
+        # peak: each part at its own dtype's peak, fp16 dense = bf16 (measured), int8 dense = 2x
+        # bf16 (B200_PROFILING.md nominal 4.5 vs 2.25 PF); the combined peak is the rate at
+        # which both parts of a pair would run back to back at those peaks:
+        #   P = f_all / (f_dist / P16 + f_sum / P8).
         tc_ns = tcw["ns"] / tcw["launches"]
         pairs_per_launch = tcw["pairs"] / tcw["launches"]
-        method_flops_per_pair = 2 * ((d + 2) + (2 * d + 1))
+        f_dist, f_sum = 2 * (d + 2), 2 * (2 * d + 1)
+        method_flops_per_pair = f_dist + f_sum
         achieved = pairs_per_launch * method_flops_per_pair / (tc_ns * 1e-9) / 1e12
         bf16 = (peaks or {}).get("bf16_tflops_sustained")
         bf16_burst = (peaks or {}).get("bf16_tflops")
-        peak = (bf16 if bf16 else 1590.0) * 1.1 / 2.25
+
+        def comb(p16):
+            return method_flops_per_pair / (f_dist / p16 + f_sum / (2.0 * p16))
+
+        peak = comb(bf16 if bf16 else 1590.0)
         roof = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
                 "traffic": traffic_from_profiles("ncu_update_tc_traffic.json"),
-                "kernel": "k_update_tc (A6 EGG-update on tcgen05, tf32)",
+                "kernel": "k_update_tc (A6 EGG-update on tcgen05: fp16 distance GEMM + exact int8 summary GEMM)",
                 "kernel_ms_per_launch": tc_ns / 1e6, "launches_per_step": tcw["launches"] / args.steps,
                 "pairs_per_step": tcw["pairs"] / args.steps,
                 "method_flops_per_pair": method_flops_per_pair,
                 "emulated_flops_per_step": tcw["flops"] / args.steps,
-                "frac_vs_burst_peak": (achieved / (bf16_burst * 1.1 / 2.25)) if bf16_burst else None,
-                "peak_basis": ("tf32 dense = MEASURED_PEAKS bf16_tflops_sustained x 1.1/2.25 (B200_PROFILING.md nominal "
-                               "ratio; sustained because the kernel is timed inside a long step)"
-                               if bf16 else "tf32 dense = fallback 1.59 PF bf16 x 1.1/2.25")}
+                "frac_vs_burst_peak": (achieved / comb(bf16_burst)) if bf16_burst else None,
+                "peak_basis": ("f_dist=2(d+2) at fp16 dense (= MEASURED_PEAKS bf16_tflops_sustained) and "
+                               "f_sum=2(2d+1) at int8 dense (2x that, B200_PROFILING.md nominal ratio), combined "
+                               "P = (f_dist+f_sum)/(f_dist/P16 + f_sum/P8); sustained because the kernel is timed "
+                               "inside a long step" if bf16 else "fallback 1.59 PF bf16, same combination")}
     else:
         # roofline of the dominant kernel (SIMT k_update): FP32 pipe
         flops_per_launch = work_flops(work, d) / iters  # per launch on this rank (its range share)

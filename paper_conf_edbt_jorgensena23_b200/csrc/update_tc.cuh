@@ -6,7 +6,7 @@
 // are computed for a tile of 128 consecutive sorted points at a time as two
 // dense contractions against "entries" (update units = cells of the hierarchy):
 //
-//   GEMM1  S[p][e] = -2 q_p . c'_e - L_e        (kind::tf32, x3 hi/lo split: ~fp32-exact)
+//   GEMM1  S[p][e] = -2 q_p . c'_e - L_e        (kind::f16, x3 hi/lo split of 2^8-scaled values)
 //          v = |q_p|^2 + S = |p - c_e|^2 - limF_e   in the tile-shifted frame
 //   classify (CUDA cores, one thread per point row of TMEM):
 //          v < 0 (sign bit)  -> entry e entirely inside the eps-ball of p (Eq.6 full part)
@@ -34,7 +34,7 @@
 //   warps 8-11  producers: thread t owns entry slot t; copies the unit's record head and
 //               digit row (block-major global layouts: coalesced along runs of units) with
 //               cp.async into the ring stage one tile ahead, then writes the origin-shifted,
-//               tf32-split GEMM1 operand row (ring of up to 8 shared-memory stages)
+//               fp16-split GEMM1 operand row (ring of up to 8 shared-memory stages)
 //   warp 12     GEMM1 issue (one thread) and TMEM owner
 //   warp 13     GEMM2 issue (one thread): decoupled from GEMM1, so a classifier group
 //               waiting on its P never holds back the next S
@@ -1315,7 +1315,7 @@ int run_planned_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr, int64_t 
       ws.tc_acc[0] += 1;
       ws.tc_acc[1] += pairs;
       ws.tc_acc[2] += padded;
-      // tensor-core operations per (point, entry) pair as executed: GEMM1 over the 3D+2 tf32
+      // tensor-core operations per (point, entry) pair as executed: GEMM1 over the 3D+2 fp16
       // operand columns (hi/lo splits), GEMM2 over the digits x (2D+1) int8 value columns
       ws.tc_pend_alg = 2LL * pairs * ((3 * D + 2) + ndig * C::NV);
       ws.tc_acc[3] += ws.tc_pend_alg;
