@@ -28,16 +28,16 @@
 // the fp32 subtree sums, as in k_update).  k_tc_expand turns each tile's ranges into a slot
 // list (one unit per entry, padded to whole entry tiles); tiles are launched heaviest-first.
 //
-// Roles (448 threads, one CTA per point tile, one CTA per SM: it owns all 512 TMEM columns):
+// Roles (512 threads, one CTA per point tile, one CTA per SM: it owns all 512 TMEM columns):
 //   warps 0-3   classifier group 0 (TMEM lanes 0..127), even entry tiles
 //   warps 4-7   classifier group 1, odd entry tiles
-//   warps 8-11  producers: thread t owns entry slot t; copies the unit's record head and
-//               digit row (block-major global layouts: coalesced along runs of units) with
-//               cp.async into the ring stage one tile ahead, then writes the origin-shifted,
-//               fp16-split GEMM1 operand row (ring of up to 8 shared-memory stages)
-//   warp 12     GEMM1 issue (one thread) and TMEM owner
-//   warp 13     GEMM2 issue (one thread): decoupled from GEMM1, so a classifier group
-//               waiting on its P never holds back the next S
+//   warps 8-11  builders: thread t owns entry slot t; from the landed record head it writes the
+//               origin-shifted, fp16-split GEMM1 operand row and the band width
+//   warp 12     MMA issue (one thread issues GEMM1 and GEMM2 in tile order) and TMEM owner
+//   warps 13-15 copy warps: fill the ring stages (up to 8) with per-lane cp.async, each warp
+//               every third entry tile, up to NST tiles ahead (the gathers by unit index are
+//               latency-bound per warp)
+// Waiting warps poll one per group and park the others in a named barrier.
 // TMEM: Q (K1 columns) | 2-3 S/P buffers of 128 columns | O (N columns, int32).
 #pragma once
 #include <cub/cub.cuh>
@@ -53,28 +53,35 @@ constexpr int kTcTile = 128;  // points per tile (TMEM lanes, GEMM M)
 constexpr int kTcEnt = 128;   // entries per entry tile (GEMM1 N, GEMM2 K)
 constexpr int kProdWarps = 4;  // producers: one entry slot per thread
 constexpr int kProd = 32 * kProdWarps;
-constexpr int kMma1Warp = 8 + kProdWarps;  // GEMM1 issue (one thread) + TMEM owner
-constexpr int kMma2Warp = kMma1Warp + 1;   // GEMM2 issue (one thread)
-constexpr int kTcThreads = (kMma2Warp + 1) * 32;  // 8 classifier + 4 producer + 2 MMA warps
+constexpr int kMmaWarp = 8 + kProdWarps;   // GEMM1 + GEMM2 issue (one thread) + TMEM owner
+constexpr int kCopyWarp0 = kMmaWarp + 1;   // stage fills by per-lane cp.async (kCopyWarps warps)
+constexpr int kCopyWarps = 3;
+constexpr int kTcThreads = (kCopyWarp0 + kCopyWarps) * 32;  // 8 classifier + 4 builder + 1 MMA + 3 copy warps
 constexpr int kTcMaxStages = 8;
 
+// |q'|^2 folded into GEMM1 (two more K columns; the classifiers read v directly) or added by
+// the classifiers (one FADD per value; K = 3D+2 keeps the stages smaller: more of them fit)
+#ifndef EGG_TC_PPFOLD
+#define EGG_TC_PPFOLD 1
+#endif
+constexpr bool kTcPP = EGG_TC_PPFOLD != 0;
 template <int D>
 struct TcCfg {
-  static constexpr int K1 = ((3 * D + 2) + 15) / 16 * 16;  // GEMM1 K (fp16): q_hi, q_lo, q_hi, s, s
-  static constexpr int QC = K1 / 2;                        // TMEM columns of Q (two fp16 per column)
+  static constexpr int KU = 3 * D + 2 + (kTcPP ? 2 : 0);  // used K columns
+  static constexpr int K1 = (KU + 15) / 16 * 16;  // GEMM1 K (fp16): q_hi, q_lo, q_hi, s, s[, pp_hi, pp_lo]
+  static constexpr int KSTEPS = K1 / 16;                  // MMA K-steps of GEMM1 (error bound of the band)
+  static constexpr int QC = (K1 / 2 + 15) / 16 * 16;      // TMEM columns of Q (two fp16 per column), 16-aligned
   static constexpr int NV = 2 * D + 1;                  // sin, cos, count
   static constexpr int DB = CellDig<D>::kBytes;         // digit row of a cell (GEMM2 N <= DB)
   static constexpr int R = CellRec<D>::kFloats;
   static constexpr int R0 = CellDig<D>::kHead;          // record head: centre, radius, count, start
-  static constexpr int R0S = (R0 / 4) % 2 == 0 ? R0 + 4 : R0;  // shared stride: conflict-free 16-B accesses
-  static constexpr int kRecBytes = kTcEnt * R0S * 4;   // record heads of a stage's entries (cp.async)
-  // shared memory: ring stages (run-time size, TcStage) | raw record heads | rare sums | misc
+  static constexpr int kRecBytes = kTcEnt * R0 * 4;   // record heads of a stage's entries, [R0/4][kTcEnt][4]
+  // shared memory: ring stages (run-time size, TcStage) | rare sums | misc
   static constexpr int SBO1 = (K1 / 8) * 128;
   static constexpr int kB1Bytes = kTcEnt * K1 * 2;
   static constexpr int kRareBytes = NV * kTcTile * 8;   // exact sums [2D][row] (2^-32) + count [row]
-  static constexpr int kSlotBytes = 4 * kTcEnt * 4;     // slot units of 4 entry tiles (producers' ring)
   static constexpr int kMiscBytes = 1024;
-  static constexpr int kFixedBytes = kRareBytes + kSlotBytes + kMiscBytes + 1024;  // +1024 alignment
+  static constexpr int kFixedBytes = kRareBytes + kMiscBytes + 1024;  // +1024 alignment
   static constexpr int kBudget = 227 * 1024;
   __host__ __device__ static constexpr int stage_bytes(int n2) {
     return (kB1Bytes + n2 * kTcEnt + kRecBytes + 8 * kTcEnt + 16 + 127) / 128 * 128;
@@ -411,8 +418,8 @@ struct TcArgs {
   const int32_t* __restrict__ g_of;
   const int32_t* __restrict__ g_cnt;
   const float* __restrict__ c_rec;
-  const int8_t* __restrict__ c_dig;   // [DB/16][cap][16] block-major digit rows
-  const float* __restrict__ c_head;   // [cap][R0] record heads
+  const int8_t* __restrict__ c_dig;   // [cap][CellDig::kStride] digit rows
+  const float* __restrict__ c_head;   // [cap][CellDig::kHeadS] record heads
   const int32_t* __restrict__ cell_of;  // unit of each sorted point
   const uint32_t* __restrict__ c_lo;
   const uint32_t* __restrict__ c_hi;
@@ -435,8 +442,8 @@ struct TcArgs {
 
 // shared-memory header of the TC kernel
 struct TcMisc {
-  uint64_t stage_full[kTcMaxStages], stage_empty[kTcMaxStages];
-  uint64_t s_full[3], p_full[3], s_free[3], o_done;
+  uint64_t stage_landed[kTcMaxStages], stage_full[kTcMaxStages], stage_empty[kTcMaxStages];
+  uint64_t s_full[3], p_full[3], o_done;
   uint32_t tbase;
   float o[kTcMaxD];
   float lo[4][kTcMaxD], hi[4][kTcMaxD];
@@ -457,8 +464,10 @@ __device__ __forceinline__ void cp_async_wait() {
 // One ring stage (run-time size: GEMM2 N = n2 depends on the digits needed):
 //   b1   [kTcEnt][K1] fp16, K-major core matrices (GEMM1 B: entry rows)            (producers)
 //   b2   [n2/16][kTcEnt][16] int8, MN-major core matrices (GEMM2 B: digits x entries) (cp.async)
-//   rec  [kTcEnt][R0S] record heads: centre (= the point of a singleton), radius, count, start (cp.async)
-//   W, cell [kTcEnt] band width and unit of every slot (-1 = padding); wmax[4]       (producers)
+//   rec  [R0/4][kTcEnt][4] record heads, block-major like c_head: centre (= the point of a
+//        singleton), radius, count, start                                              (TMA)
+//   W [kTcEnt] band width of every slot, wmax[4]                                       (builders)
+//   cell [kTcEnt] unit of every slot (-1 = padding): the tile's slot list              (TMA)
 template <int D>
 struct TcStage {
   float* b1;
@@ -478,16 +487,11 @@ struct TcStage {
     cell = reinterpret_cast<int32_t*>(m + 4 * kTcEnt);
     wmax = reinterpret_cast<float*>(m + 8 * kTcEnt);
   }
-  __device__ int32_t cnt(int e) const { return __float_as_int(rec[e * TcCfg<D>::R0S + D + 1]); }
-  __device__ int32_t start(int e) const { return __float_as_int(rec[e * TcCfg<D>::R0S + D + 2]); }
-  __device__ float pt(int e, int i) const { return rec[e * TcCfg<D>::R0S + i]; }
+  __device__ float hf(int e, int i) const { return rec[((i >> 2) * kTcEnt + e) * 4 + (i & 3)]; }
+  __device__ int32_t cnt(int e) const { return __float_as_int(hf(e, D + 1)); }
+  __device__ int32_t start(int e) const { return __float_as_int(hf(e, D + 2)); }
+  __device__ float pt(int e, int i) const { return hf(e, i); }
 };
-
-// record head field i (centre 0..D-1, radius D, count D+1, start D+2) of unit c (block-major)
-template <int D>
-__device__ __forceinline__ float head_f(const float* __restrict__ c_head, int64_t cap, int32_t c, int i) {
-  return c_head[((int64_t)(i >> 2) * cap + c) * 4 + (i & 3)];
-}
 
 // Exact path for a multi-point unit e inside the band of point pe (P stays 0 for the pair):
 // refine with the unit's exact MBR, then its points one by one (fp32 + fp64 re-decision as
@@ -547,74 +551,85 @@ constexpr float kTcScale2 = 65536.f;
 
 template <int D>
 __device__ __forceinline__ float tc_build_entry(const TcArgs<D>& a, const float (&o)[D],
-                                                const TcStage<D>& st, int pt, int32_t c,
-                                                const float* __restrict__ rec, float Rq, float Rqi) {
+                                                const TcStage<D>& st, int pt, int32_t c, float Rq, float Rqi) {
+  // branchless: a padding slot computes on whatever its record holds and selects the padding
+  // row at the end
   using C = TcCfg<D>;
   constexpr int K1 = C::K1;
-  float b[K1];
-  float W = 0.f;
-  if (c >= 0) {
-    float r[C::R0];
-    const float4* r4 = reinterpret_cast<const float4*>(rec);  // staged by cp.async
+  const bool real = c >= 0;
+  float r[C::R0];
+  const float4* r4 = reinterpret_cast<const float4*>(st.rec);  // landed by cp.async, block-major
 #pragma unroll
-    for (int k = 0; k < C::R0 / 4; ++k) {
-      const float4 t4 = r4[k];
-      r[4 * k] = t4.x;
-      r[4 * k + 1] = t4.y;
-      r[4 * k + 2] = t4.z;
-      r[4 * k + 3] = t4.w;
-    }
-    float cc0 = 0.f, cc1 = 0.f, cinf = 0.f;  // two independent chains (latency)
+  for (int k = 0; k < C::R0 / 4; ++k) {
+    const float4 t4 = r4[k * kTcEnt + pt];
+    r[4 * k] = t4.x;
+    r[4 * k + 1] = t4.y;
+    r[4 * k + 2] = t4.z;
+    r[4 * k + 3] = t4.w;
+  }
+  __half hb[K1];  // B1 row: c'_hi, c'_hi, c'_lo, -L_hi, -L_lo, 2^8, 2^8, 0... (A carries the -2)
+  float cc0 = 0.f, cc1 = 0.f, cinf = 0.f;  // two independent chains (latency)
 #pragma unroll
-    for (int i = 0; i < D; ++i) {
-      const float cp = r[i] - o[i];
-      float h, l;
-      tc::split_h(cp * kTcScale, h, l);
-      b[i] = -2.f * h;
-      b[D + i] = -2.f * h;
-      b[2 * D + i] = -2.f * l;
-      if (i & 1) cc1 = fmaf(cp, cp, cc1);
-      else cc0 = fmaf(cp, cp, cc0);
-      cinf = fmaxf(cinf, fabsf(cp));
-    }
-    const float cc = cc0 + cc1;
-    const float rad = r[D];
-    // error budget: eta = rounding of the shifted frame; E bounds |v - v_exact|:
-    //   fp16 split of -2 q.c' (round-to-nearest hi, lo rounded again, lo*lo dropped):
-    //     <= 2 * 3 * 2^-22 sum|q_i||c'_i| <= 2^-19.4 |q||c'|               (Cauchy-Schwarz)
-    //   tensor-core accumulation, 2 K-steps of 16 products + accumulator, each truncating
-    //     <= 17 * 2^-23 of the sum of |terms| (2|q||c'| + |L|):  <= 2^-16.9 |q||c'| + 2^-17.9 |L|
-    //   L = limF - |c'|^2 split hi/lo (2^-22 |L|); fp32 |q|^2, |c'|^2 (D FMAs): (D+2) u (|q|^2 + cc)
-    //   => E <= 2^-16 Rq|c'| + 2^-17 |L| + 2^-20 (Rq^2 + cc)   (Rq >= |q|, D <= 12); unscaled
-    const float eta = 2.5f * kU * sqrtf((float)D) * (Rqi + cinf);
-    const float ep = (a.e + rad) * (1.f + 8.f * kU) + eta;
-    const float em = (a.e - rad) * (1.f - 8.f * kU) - eta;
-    const float limF0 = em > 0.f ? em * em * (1.f - 4.f * kU) : -1.f;
-    const float E = 1.52587890625e-05f * (Rq * sqrtf(cc)) + 7.62939453125e-06f * fabsf(limF0 - cc) +
-                    9.5367431640625e-07f * (cc + Rq * Rq) + 1e-30f;
-    const float limF = em > 0.f ? limF0 - E : -1.f;
-    const float limO = ep * ep * (1.f + 4.f * kU) + E;
-    W = (limO - limF) * (1.f + 4.f * kU) * kTcScale2;  // in the scaled units of v
-    const float L = limF - cc;
-    float Lh, Ll;
-    tc::split_h(L * kTcScale, Lh, Ll);  // times A's s = 2^8 column: L * 2^16
-    b[3 * D] = -Lh;
-    b[3 * D + 1] = -Ll;
-  } else {
-#pragma unroll
-    for (int k = 0; k < 3 * D + 2; ++k) b[k] = 0.f;
-    b[3 * D] = 60000.f;  // v = 2^8 * 60000: far outside, never ambiguous
+  for (int i = 0; i < D; ++i) {
+    const float cp = r[i] - o[i];
+    const float x = cp * kTcScale;
+    const __half h = __float2half_rn(x);
+    const __half l = __float2half_rn(x - __half2float(h));
+    hb[i] = h;
+    hb[D + i] = h;
+    hb[2 * D + i] = l;
+    if (i & 1) cc1 = fmaf(cp, cp, cc1);
+    else cc0 = fmaf(cp, cp, cc0);
+    cinf = fmaxf(cinf, fabsf(cp));
+  }
+  const float cc = cc0 + cc1;
+  const float rad = r[D];
+  // error budget: eta = rounding of the shifted frame; E bounds |v - v_exact|:
+  //   fp16 split of -2 q.c' (round-to-nearest hi, lo rounded again, lo*lo dropped):
+  //     <= 2 * 3 * 2^-22 sum|q_i||c'_i| <= 2^-19.4 |q||c'|               (Cauchy-Schwarz)
+  //   tensor-core accumulation, KSTEPS K-steps of 16 products + accumulator, each truncating
+  //     <= 17 * 2^-23 of the sum of |terms| (2|q||c'| + |L| + |q|^2): acc = KSTEPS * 17 * 2^-23
+  //   L = limF - |c'|^2 and |q|^2 split hi/lo (2^-22 each); fp32 |q|^2, |c'|^2 (D FMAs):
+  //     (D+2) u (|q|^2 + cc) <= 2^-20 (|q|^2 + cc)
+  //   => E <= (2^-19.4 + 2 acc) Rq|c'| + (2^-22 + acc)(|L| + Rq^2) + 2^-20 (Rq^2 + cc)
+  //      (Rq >= |q|, D <= 12); coefficients rounded up by 1%; unscaled
+  const float eta = 2.5f * kU * sqrtf((float)D) * (Rqi + cinf);
+  const float ep = (a.e + rad) * (1.f + 8.f * kU) + eta;
+  const float em = (a.e - rad) * (1.f - 8.f * kU) - eta;
+  const float limF0 = em > 0.f ? em * em * (1.f - 4.f * kU) : -1.f;
+  constexpr float acc = (float)C::KSTEPS * 17.f * 1.1920928955078125e-07f;
+  constexpr float e1 = 1.01f * (1.4505753e-06f + 2.f * acc);  // 2^-19.4 = 6 * 2^-22
+  constexpr float e2 = 1.01f * (2.384185791015625e-07f + acc);
+  const float E = e1 * (Rq * sqrtf(cc)) + e2 * (fabsf(limF0 - cc) + Rq * Rq) +
+                  9.5367431640625e-07f * (cc + Rq * Rq) + 1e-30f;
+  const float limF = em > 0.f ? limF0 - E : -1.f;
+  const float limO = ep * ep * (1.f + 4.f * kU) + E;
+  const float W = real ? (limO - limF) * (1.f + 4.f * kU) * kTcScale2 : 0.f;  // in the scaled units of v
+  const float xL = -(limF - cc) * kTcScale;  // times A's s = 2^8 column: -L * 2^16
+  const __half Lh = __float2half_rn(xL);
+  hb[3 * D] = Lh;
+  hb[3 * D + 1] = __float2half_rn(xL - __half2float(Lh));
+  if constexpr (kTcPP) {
+    hb[3 * D + 2] = __float2half_rn(kTcScale);  // times A's 2^8-scaled |q'|^2 halves: + |q'|^2 * 2^16
+    hb[3 * D + 3] = __float2half_rn(kTcScale);
   }
 #pragma unroll
-  for (int k = 3 * D + 2; k < K1; ++k) b[k] = 0.f;
-  // B1: K-major fp16, entry rows (8 K-values per 16-byte core-matrix row)
-  {
-    unsigned char* b1 = reinterpret_cast<unsigned char*>(st.b1) + (pt >> 3) * C::SBO1 + (pt & 7) * 16;
+  for (int k = C::KU; k < K1; ++k) hb[k] = __float2half_rn(0.f);
+  if (!real) {  // padding: v = 2^8 * 60000 + |q'|^2 2^16, far outside, never ambiguous (selects)
 #pragma unroll
-    for (int kc = 0; kc < K1 / 8; ++kc)
-      *reinterpret_cast<uint4*>(b1 + kc * 128) =
-          make_uint4(tc::pack_h2(b[8 * kc], b[8 * kc + 1]), tc::pack_h2(b[8 * kc + 2], b[8 * kc + 3]),
-                     tc::pack_h2(b[8 * kc + 4], b[8 * kc + 5]), tc::pack_h2(b[8 * kc + 6], b[8 * kc + 7]));
+    for (int k = 0; k < 3 * D + 2; ++k) hb[k] = __float2half_rn(k == 3 * D ? 60000.f : 0.f);
+  }
+  // B1: K-major fp16, entry rows (8 K-values per 16-byte core-matrix row)
+  unsigned char* b1 = reinterpret_cast<unsigned char*>(st.b1) + (pt >> 3) * C::SBO1 + (pt & 7) * 16;
+#pragma unroll
+  for (int kc = 0; kc < K1 / 8; ++kc) {
+    uint32_t w[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+      const __half2 h2 = __halves2half2(hb[8 * kc + 2 * q], hb[8 * kc + 2 * q + 1]);
+      w[q] = *reinterpret_cast<const uint32_t*>(&h2);
+    }
+    *reinterpret_cast<uint4*>(b1 + kc * 128) = make_uint4(w[0], w[1], w[2], w[3]);
   }
   st.W[pt] = W;
   return W;
@@ -664,8 +679,7 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
   const int NST = a.nst, NS = a.ns, SB = a.stage_bytes, N2 = a.n2;
   unsigned char* ring = tsm;
   unsigned long long* rare = reinterpret_cast<unsigned long long*>(tsm + (size_t)NST * SB);
-  int32_t* slots = reinterpret_cast<int32_t*>(tsm + (size_t)NST * SB + C::kRareBytes);
-  TcMisc* ms = reinterpret_cast<TcMisc*>(tsm + (size_t)NST * SB + C::kRareBytes + C::kSlotBytes);
+  TcMisc* ms = reinterpret_cast<TcMisc*>(tsm + (size_t)NST * SB + C::kRareBytes);
 
   const int tid = threadIdx.x, wid = tid >> 5, lane = tid & 31;
   const int64_t tile = a.perm[blockIdx.x];  // heaviest point tiles first (shorter tail)
@@ -674,24 +688,24 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
   const int T = (ne + kTcEnt - 1) / kTcEnt;  // entry tiles (the slot list is padded to T * kTcEnt)
   const int kColS = C::QC, kColO = C::QC + NS * kTcEnt;
 #ifdef EGG_TC_PROF
-  unsigned long long prof_acc[4] = {0, 0, 0, 0};
+  unsigned long long prof_acc[6] = {0, 0, 0, 0, 0, 0};
 #endif
 
   // ---- setup -------------------------------------------------------------------------
   if (tid == 0) {
     for (int s = 0; s < NST; ++s) {
-      tc::bar_init(&ms->stage_full[s], kProd);
+      tc::bar_init(&ms->stage_landed[s], 32);    // one cp.async-completion arrival per copy lane
+      tc::bar_init(&ms->stage_full[s], kProd);   // one arrival per builder thread (entry slot)
       tc::bar_init(&ms->stage_empty[s], 1);
     }
     for (int b = 0; b < NS; ++b) {
       tc::bar_init(&ms->s_full[b], 1);
       tc::bar_init(&ms->p_full[b], kTcTile);
-      tc::bar_init(&ms->s_free[b], 1);
     }
     tc::bar_init(&ms->o_done, 1);
     tc::bar_fence_init();
   }
-  if (wid == kMma1Warp) tc::tmem_alloc<512>(&ms->tbase);
+  if (wid == kMmaWarp) tc::tmem_alloc<512>(&ms->tbase);
   for (int t = tid; t < NV * kTcTile; t += kTcThreads) rare[t] = 0ull;
 
   // classifier rows: every classifier thread holds its point
@@ -729,7 +743,7 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
     ms->Rqi = 0.f;
   }
   __syncthreads();
-  float pp = 3.0e38f;  // |q|^2 (invalid rows never classify inside or ambiguous)
+  float pp = 3.0e38f;  // |q'|^2 (invalid rows never classify inside or ambiguous)
   if (is_cls) {
     float q[D];
     float s = 0.f, rinf = 0.f;
@@ -739,7 +753,7 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
       s = fmaf(q[i], q[i], s);
       rinf = fmaxf(rinf, fabsf(q[i]));
     }
-    if (valid) pp = s * kTcScale2;  // v is formed in the scaled units of GEMM1
+    if (valid) pp = s * kTcScale2;  // (!kTcPP) v = S + |q'|^2, in the scaled units of GEMM1
     if (grp == 0) {
       float r2 = sqrtf(s) * (1.f + 4.f * kU), ri = rinf;
 #pragma unroll
@@ -754,17 +768,27 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
       // Q row -> TMEM columns [0, K1/2) as fp16 pairs (scaled by 2^8): q_hi, q_lo, q_hi, s, s, 0...
       float v[K1];
 #pragma unroll
-      for (int i = 0; i < D; ++i) {
+      for (int i = 0; i < D; ++i) {  // -2 q' halves (exact scaling): B carries c' unscaled
         float h, l;
         tc::split_h(q[i] * kTcScale, h, l);
-        v[i] = h;
-        v[D + i] = l;
-        v[2 * D + i] = h;
+        v[i] = -2.f * h;
+        v[D + i] = -2.f * l;
+        v[2 * D + i] = -2.f * h;
       }
       v[3 * D] = kTcScale;
       v[3 * D + 1] = kTcScale;
+      // |q'|^2 (scaled by 2^8; B's 2^8 columns make it |q'|^2 * 2^16 in v): the GEMM forms
+      // v = |p - c_e|^2 - limF_e directly.  Invalid rows: 60000 * 2^8, never inside or ambiguous.
+      if constexpr (kTcPP) {
+        if (valid) {
+          tc::split_h(s * kTcScale, v[3 * D + 2], v[3 * D + 3]);
+        } else {
+          v[3 * D + 2] = 60000.f;
+          v[3 * D + 3] = 0.f;
+        }
+      }
 #pragma unroll
-      for (int k = 3 * D + 2; k < K1; ++k) v[k] = 0.f;
+      for (int k = C::KU; k < K1; ++k) v[k] = 0.f;
       const uint32_t taddr = ms->tbase + ((uint32_t)(32 * (wid & 3)) << 16);
 #pragma unroll
       for (int c = 0; c < K1 / 16; ++c) {
@@ -782,137 +806,137 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
   const uint32_t tb = ms->tbase;
 
   if (wid >= 8 && wid < 8 + kProdWarps) {
-    // ================================ producers ================================
-    // Thread pt owns entry slot pt of every entry tile.  The unit of slot pt of tile t comes
-    // from the slot list (k_tc_expand).  (Walking the range list in the kernel instead was
-    // measured slower: its index work sits on the producers' critical path.)
+    // ================================ builders ================================
+    // Thread pt builds entry slot pt of every entry tile from the record head the copy warp
+    // landed: the origin-shifted, fp16-split GEMM1 operand row and the band width W.
     const int pt = tid - 256;  // entry slot 0..127
-    const int pw = pt >> 5;
     const float Rq = ms->Rq, Rqi = ms->Rqi;
     float ov[D];  // tile origin, in registers for the operand builds
 #pragma unroll
     for (int i = 0; i < D; ++i) ov[i] = ms->o[i];
-    const int nchunk = N2 / 16;
-    const int32_t* __restrict__ ent = a.ent + a.eoff[tile];
-    // copies of entry tile t into its stage (one cp.async group per tile, empty beyond T)
-    // Per entry tile t: the slot's unit (slot list, one tile ahead), then its record head (the
-    // 16-byte blocks of the block-major c_head: coalesced along a run of units) and digit row
-    // by cp.async straight into the stage, one tile ahead of the build.
-    constexpr int NH = R0 / 4;
-    // slot units are copied (cp.async, 4 bytes) three tiles ahead into a per-thread ring in
-    // shared memory, so the slot list's DRAM latency never sits in front of a fetch
-    int32_t* slotq = slots + pt;  // [4][kProd]: slot of tile t at slotq[(t & 3) * kProd]
-    auto slot_copy = [&](int t) {
-      if (t < T) {
-        asm volatile("cp.async.ca.shared.global [%0], [%1], 4;" ::"r"(tc::smem_addr(slotq + (t & 3) * kProd)),
-                     "l"(ent + (int64_t)t * kTcEnt + pt)
-                     : "memory");
-      }
-    };
-    RingPos fp;  // stage of the tile being fetched
-    auto fetch = [&](int t) {  // copies for tile t (cp.async group, possibly empty); slot of t landed
-      if (t < T) {
-        const int32_t c = slotq[(t & 3) * kProd];
-        TCP_T(f0);
-        if (t >= NST) tc::bar_sleep(&ms->stage_empty[fp.i], fp.ph ^ 1u);
-        TCP_T(f1);
-        TCP_ADD(3, f1 - f0);
-        TcStage<D> st(ring, fp.i, SB, N2);
-        st.cell[pt] = c;
-        if (c >= 0) {
-          float* dst = st.rec + pt * C::R0S;
-#pragma unroll
-          for (int k = 0; k < NH; ++k) cp_async16(dst + 4 * k, a.c_head + ((int64_t)k * a.cap + c) * 4);
-          int8_t* b2 = st.b2 + pt * 16;
-          const int8_t* dg = a.c_dig + (int64_t)c * 16;
-#pragma unroll
-          for (int k = 0; k < C::DB / 16; ++k)
-            if (k < nchunk) cp_async16(b2 + k * (16 * kTcEnt), dg + (int64_t)k * a.cap * 16);
-        }
-        fp.adv(NST);
-      }
-    };
-    // prologue: slots of tiles 0..2, then tile 0's copies (group 0 also carries slot 3)
-    slot_copy(0);
-    slot_copy(1);
-    slot_copy(2);
-    cp_async_commit();
-    cp_async_wait<0>();
-    fetch(0);
-    slot_copy(3);
-    cp_async_commit();
-    RingPos bp;  // stage of the tile being built
+    RingPos bp;
     for (int jt = 0; jt < T; ++jt) {
       TCP_T(p0);
-      fetch(jt + 1);                // next tile's copies in flight during this build
-      slot_copy(jt + 4);
-      cp_async_commit();
+      if (wid == 8) tc::bar_poll(&ms->stage_landed[bp.i], bp.ph);
+      tc::named_sync(3, kProd);
       TCP_T(p1);
-      TCP_ADD(0, p1 - p0);
-      cp_async_wait<1>();           // this tile's record heads and digit rows (and slot jt+3) landed
-      TCP_T(p2);
-      TCP_ADD(1, p2 - p1);
       TcStage<D> st(ring, bp.i, SB, N2);
-      const float W = tc_build_entry<D>(a, ov, st, pt, st.cell[pt], st.rec + pt * C::R0S, Rq, Rqi);
+      const float W = tc_build_entry<D>(a, ov, st, pt, st.cell[pt], Rq, Rqi);
       // chunk maximum of the band widths (W >= 0: its bits order as unsigned integers)
       const uint32_t wm = __reduce_max_sync(FULLMASK, __float_as_uint(W));
-      if (lane == 0) st.wmax[pw] = __uint_as_float(wm);
+      if (lane == 0) st.wmax[pt >> 5] = __uint_as_float(wm);
       tc::fence_proxy_async();
       tc::bar_arrive(&ms->stage_full[bp.i]);
       bp.adv(NST);
-      TCP_T(p3);
-      TCP_ADD(2, p3 - p2);
+      TCP_T(p2);
+      TCP_ADD(0, p1 - p0);
+      TCP_ADD(1, p2 - p1);
     }
   }
 
-  if (wid == kMma1Warp && lane == 0) {
-    // ================================ GEMM1 issue ================================
-    // S[jt % NS] = Q . B1(jt)^T once stage jt is built and GEMM2(jt - NS) released the buffer.
-    constexpr uint32_t id1 = tc::idesc_f16(128, kTcEnt);
-    const uint32_t ring_s = tc::smem_addr(ring);
-    RingPos sp, bq;
-    for (int jt = 0; jt < T; ++jt) {
-      const int s = sp.i, b = bq.i;
-      TCP_T(m0);
-      tc::bar_sleep(&ms->stage_full[s], sp.ph);
-      TCP_T(m1);
-      if (jt >= NS) tc::bar_sleep(&ms->s_free[b], bq.ph ^ 1u);
-      TCP_T(m2);
-      TCP_ADD(0, m1 - m0);
-      TCP_ADD(1, m2 - m1);
-      tc::fence_after();
-      const uint32_t b1 = ring_s + s * SB;
+  if (wid >= kCopyWarp0) {
+    // ================================ copy warps ================================
+    // Copy warp w fills the stages of entry tiles t = w mod kCopyWarps (several warps: the
+    // gathers by unit index are latency-bound per warp), up to NST tiles ahead: the tile's 128
+    // slot units (512 B of the slot list) and, for slot e = lane + 32 j, its record head and
+    // digit row by 16-byte cp.async (block-major global layouts: consecutive lanes read
+    // consecutive units of a run, so the copies coalesce).  Each lane's completion arrives on
+    // stage_landed (cp.async.mbarrier.arrive.noinc); the warps never wait for their copies.
+    constexpr int NH = R0 / 4;
+    const int nchunk = N2 / 16;
+    const int cw = wid - kCopyWarp0;
+    const int32_t* __restrict__ ent = a.ent + a.eoff[tile];  // 512-byte aligned (padded tiles)
+    const char* __restrict__ hb = reinterpret_cast<const char*>(a.c_head);
+    const char* __restrict__ db = reinterpret_cast<const char*>(a.c_dig);
+    const int64_t capB = a.cap * 16;  // bytes of one 16-byte block column
+    int cn[4];
 #pragma unroll
-      for (int k = 0; k < K1 / 16; ++k)  // 16 fp16 K-values per MMA: 8 TMEM columns of A, 2 core matrices of B
-        tc::mma_ts_f16(tb + kColS + kTcEnt * b, tb + 8 * k, tc::sdesc(b1 + k * 256, 128, C::SBO1), id1, k > 0);
-      tc::mma_commit(&ms->s_full[b]);
-      sp.adv(NST);
-      bq.adv(NS);
+    for (int j = 0; j < 4; ++j) cn[j] = cw < T ? ent[(int64_t)cw * kTcEnt + lane + 32 * j] : -1;
+    RingPos fp;
+    for (int k = 0; k < cw; ++k) fp.adv(NST);
+    for (int t = cw; t < T; t += kCopyWarps) {
+      int cu[4];
+#pragma unroll
+      for (int j = 0; j < 4; ++j) cu[j] = cn[j];
+      if (t + kCopyWarps < T) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) cn[j] = ent[(int64_t)(t + kCopyWarps) * kTcEnt + lane + 32 * j];
+      }
+      TCP_T(f0);
+      if (t >= NST) {
+        if (lane == 0) tc::bar_poll(&ms->stage_empty[fp.i], fp.ph ^ 1u);
+        __syncwarp();
+      }
+      TCP_T(f1);
+      TcStage<D> st(ring, fp.i, SB, N2);
+      cp_async16(st.cell + 4 * lane, ent + (int64_t)t * kTcEnt + 4 * lane);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) {
+        const int c = cu[j];
+        if (c >= 0) {
+          const int e = lane + 32 * j;
+          const char* hs = hb + (int64_t)c * 16;
+#pragma unroll
+          for (int k = 0; k < NH; ++k) cp_async16(st.rec + ((size_t)k * kTcEnt + e) * 4, hs + k * capB);
+          const char* ds = db + (int64_t)c * 16;
+          int8_t* dd = st.b2 + e * 16;
+#pragma unroll
+          for (int k = 0; k < C::DB / 16; ++k)
+            if (k < nchunk) cp_async16(dd + k * (16 * kTcEnt), ds + k * capB);
+        }
+      }
+      asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(tc::smem_addr(&ms->stage_landed[fp.i]))
+                   : "memory");
+#pragma unroll
+      for (int k = 0; k < kCopyWarps; ++k) fp.adv(NST);
+      TCP_T(f2);
+      if (cw == 0) {
+        TCP_ADD(0, f2 - f1);
+        TCP_ADD(1, f1 - f0);
+      }
     }
+    cp_async_wait<0>();
   }
-  if (wid == kMma2Warp && lane == 0) {
-    // ================================ GEMM2 issue ================================
-    // O += P . B2(jt)^T (int8 x int8 -> int32, exact) once a classifier group wrote P(jt)
-    // into the first 32 columns of S[jt % NS]; releases the stage and the S buffer.
+
+  if (wid == kMmaWarp && lane == 0) {
+    // ================================ MMA issue ================================
+    // One thread issues both GEMMs in tile order: GEMM1(g1) = Q . B1(g1)^T into S[g1 % NS]
+    // once stage g1 is built and GEMM2(g1 - NS) has been issued (same-thread tcgen05.mma run
+    // in issue order, so that GEMM2 has read P before GEMM1 overwrites the buffer); GEMM2(g2):
+    // O += P(g2) . B2(g2)^T (int8 x int8 -> int32, exact) once a classifier group wrote P.
+    constexpr uint32_t id1 = tc::idesc_f16(128, kTcEnt);
     const uint32_t id2 = tc::idesc_s8(128, N2, true);
     const uint32_t ring_s = tc::smem_addr(ring);
-    RingPos sp, bq;
-    for (int jt = 0; jt < T; ++jt) {
-      const int s = sp.i, b = bq.i;
-      TCP_T(m0);
-      tc::bar_sleep(&ms->p_full[b], bq.ph);
-      TCP_T(m1);
-      TCP_ADD(0, m1 - m0);
-      tc::fence_after();
-      const uint32_t b2 = ring_s + s * SB + C::kB1Bytes;
+    RingPos s1, b1q, s2, b2q;
+    int g1 = 0, g2 = 0;
+    while (g2 < T) {
+      bool did = false;
+      if (g1 < T && g1 - g2 < NS && tc::bar_test(&ms->stage_full[s1.i], s1.ph)) {
+        tc::fence_after();
+        const uint32_t b1 = ring_s + s1.i * SB;
 #pragma unroll
-      for (int k = 0; k < kTcEnt / 32; ++k)
-        tc::mma_ts_s8(tb + kColO, tb + kColS + kTcEnt * b + 8 * k, tc::sdesc(b2 + k * 512, 128, 16 * kTcEnt), id2,
-                      (jt > 0) || (k > 0));
-      tc::mma_commit(&ms->stage_empty[s]);
-      tc::mma_commit(&ms->s_free[b]);
-      sp.adv(NST);
-      bq.adv(NS);
+        for (int k = 0; k < K1 / 16; ++k)  // 16 fp16 K-values per MMA: 8 TMEM columns of A, 2 core matrices of B
+          tc::mma_ts_f16(tb + kColS + kTcEnt * b1q.i, tb + 8 * k, tc::sdesc(b1 + k * 256, 128, C::SBO1), id1, k > 0);
+        tc::mma_commit(&ms->s_full[b1q.i]);
+        s1.adv(NST);
+        b1q.adv(NS);
+        ++g1;
+        did = true;
+      }
+      if (g2 < g1 && tc::bar_test(&ms->p_full[b2q.i], b2q.ph)) {
+        tc::fence_after();
+        const uint32_t b2 = ring_s + s2.i * SB + C::kB1Bytes;
+#pragma unroll
+        for (int k = 0; k < kTcEnt / 32; ++k)
+          tc::mma_ts_s8(tb + kColO, tb + kColS + kTcEnt * b2q.i + 8 * k, tc::sdesc(b2 + k * 512, 128, 16 * kTcEnt), id2,
+                        (g2 > 0) || (k > 0));
+        tc::mma_commit(&ms->stage_empty[s2.i]);
+        s2.adv(NST);
+        b2q.adv(NS);
+        ++g2;
+        did = true;
+      }
+      if (!did) __nanosleep(20);
     }
     tc::mma_commit(&ms->o_done);
   }
@@ -920,45 +944,48 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
   if (is_cls) {
     // ================================ classifiers ================================
     const uint32_t lane_off = (uint32_t)(32 * (wid & 3)) << 16;
-    const int Tg = grp ? T / 2 : (T + 1) / 2;
     const float lim_in = a.e2f * (1.f - a.rel), lim_out = a.e2f * (1.f + a.rel);
     RingPos sp, bq;  // stage / S buffer of tile jt = 2 kk + grp
     if (grp) {
       sp.adv(NST);
       bq.adv(NS);
     }
-    for (int kk = 0; kk < Tg; ++kk) {
+    for (int jt = grp; jt < T; jt += 2) {
       const int s = sp.i, b = bq.i;
       TcStage<D> st(ring, s, SB, N2);
       TCP_T(c0);
-      tc::bar_sleep(&ms->s_full[b], bq.ph);
+      // one polling warp per group; the other three sleep in the group's named barrier (the
+      // poller's acquire + the barrier order their TMEM reads after the MMA, with fence_after)
+      if ((wid & 3) == 0) tc::bar_poll(&ms->s_full[b], bq.ph);
+      tc::named_sync(1 + grp, kTcTile);
       TCP_T(c1);
       TCP_ADD(0, c1 - c0);
       tc::fence_after();
       const uint32_t sb = tb + lane_off + kColS + kTcEnt * b;
-#pragma unroll 1
-      for (int cp = 0; cp < kTcEnt / 64; ++cp) {
-        uint32_t v[2][32];
-        tc::ld32(sb + 64 * cp, v[0]);
-        tc::ld32(sb + 64 * cp + 32, v[1]);
-        TCP_T(l0);
-        tc::wait_ld();
-        TCP_T(l1);
-        TCP_ADD(1, l1 - l0);
-        uint32_t pw[16];
+      // four chunks of 32 entries, software-pipelined: the TMEM load of chunk c+1 is in flight
+      // while chunk c is classified
+      uint32_t v[2][32];
+      tc::ld32(sb, v[0]);
+      TCP_T(l0);
+      tc::wait_ld_regs(v[0]);
+      TCP_T(l1);
+      TCP_ADD(1, l1 - l0);
 #pragma unroll
-        for (int h = 0; h < 2; ++h) {
-          const int c = 2 * cp + h;
+      for (int c = 0; c < kTcEnt / 32; ++c) {
+        const int h = c & 1;
+        if (c + 1 < kTcEnt / 32) tc::ld32(sb + 32 * (c + 1), v[h ^ 1]);
+        uint32_t pw[8];
+        {
           const uint32_t wm = __float_as_uint(st.wmax[c]);
           uint32_t mn = 0xFFFFFFFFu;
 #pragma unroll
           for (int jx = 0; jx < 32; ++jx) {
-            v[h][jx] = __float_as_uint(__uint_as_float(v[h][jx]) + pp);  // |p - c_e|^2 - limF_e
+            if constexpr (!kTcPP) v[h][jx] = __float_as_uint(__uint_as_float(v[h][jx]) + pp);  // |p-c|^2 - limF
             mn = min(mn, v[h][jx]);  // unsigned: negative values (inside) compare large
           }
 #pragma unroll
           for (int w = 0; w < 8; ++w)
-            pw[8 * h + w] = sign_bytes4(v[h][4 * w], v[h][4 * w + 1], v[h][4 * w + 2], v[h][4 * w + 3]);
+            pw[w] = sign_bytes4(v[h][4 * w], v[h][4 * w + 1], v[h][4 * w + 2], v[h][4 * w + 3]);
           TCP_T(b0);
           if (mn < wm) {  // some pair of this chunk may lie in a band (0 <= f <= max W): exact decisions
             uint32_t bm = 0u;
@@ -1000,14 +1027,15 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
 #pragma unroll
             for (int w = 0; w < 8; ++w) {
               const uint32_t f4 = (fm >> (4 * w)) & 0xFu;
-              pw[8 * h + w] |= (f4 & 1u ? 0xFFu : 0u) | (f4 & 2u ? 0xFF00u : 0u) | (f4 & 4u ? 0xFF0000u : 0u) |
-                               (f4 & 8u ? 0xFF000000u : 0u);
+              pw[w] |= (f4 & 1u ? 0xFFu : 0u) | (f4 & 2u ? 0xFF00u : 0u) | (f4 & 4u ? 0xFF0000u : 0u) |
+                       (f4 & 8u ? 0xFF000000u : 0u);
             }
           }
           TCP_T(b1);
           TCP_ADD(2, b1 - b0);
         }
-        tc::st16(sb + 16 * cp, pw);  // P (int8, -1 = inside) over S columns already read
+        tc::st8(sb + 8 * c, pw);  // P (int8, -1 = inside) over S columns 0..31, already read
+        if (c + 1 < kTcEnt / 32) tc::wait_ld_regs(v[h ^ 1]);
       }
       TCP_T(w0);
       tc::wait_st();
@@ -1027,10 +1055,11 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
     int slot = -1;
     if (tid == 0 || tid == 128) slot = 0;
     else if (tid == 256) slot = 4;
-    else if (wid == kMma1Warp && lane == 0) slot = 8;
-    else if (wid == kMma2Warp && lane == 0) slot = 12;
-    if (slot >= 0 && a.prof)
-      for (int k = 0; k < (slot == 12 ? 1 : 4); ++k) atomicAdd(&a.prof[slot + k], prof_acc[k]);
+    else if (wid == kCopyWarp0 && lane == 0) slot = 10;
+    if (slot >= 0 && a.prof) {
+      const int nk = slot == 12 ? 1 : slot == 0 ? 4 : 2;
+      for (int k = 0; k < nk; ++k) atomicAdd(&a.prof[slot + k], prof_acc[k]);
+    }
     if (tid == 0 && a.prof) atomicAdd(&a.prof[15], (unsigned long long)T);
   }
 #endif
@@ -1084,7 +1113,7 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
   }
   tc::fence_before();
   __syncthreads();
-  if (wid == kMma1Warp) {
+  if (wid == kMmaWarp) {
     tc::fence_after();
     tc::tmem_dealloc<512>(tb);
   }
@@ -1263,7 +1292,8 @@ int run_planned_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr, int64_t 
     const int sbytes = C::stage_bytes(n2);
     int nst = (C::kBudget - C::kFixedBytes) / sbytes;
     nst = nst > kTcMaxStages ? kTcMaxStages : nst;
-    if (nst < 2 || C::QC + 2 * kTcEnt + n2 > 512) {  // cannot happen for D <= kTcMaxD
+    // >= 3 stages: a worker group builds its next tile (jt + 2) before classifying jt
+    if (nst < 3 || C::QC + 2 * kTcEnt + n2 > 512) {  // cannot happen for D <= kTcMaxD
       ws.tc_used = 0;
       return run_update_simt<D>(ws, lo, hi, nbr);
     }
@@ -1317,7 +1347,7 @@ int run_planned_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr, int64_t 
       ws.tc_acc[2] += padded;
       // tensor-core operations per (point, entry) pair as executed: GEMM1 over the 3D+2 fp16
       // operand columns (hi/lo splits), GEMM2 over the digits x (2D+1) int8 value columns
-      ws.tc_pend_alg = 2LL * pairs * ((3 * D + 2) + ndig * C::NV);
+      ws.tc_pend_alg = 2LL * pairs * (C::KU + ndig * C::NV);
       ws.tc_acc[3] += ws.tc_pend_alg;
       EGG_CUDA(cudaEventRecord(ws.tc_ev[0], ws.stream));
     }
@@ -1339,10 +1369,10 @@ int run_planned_tc(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr, int64_t 
       EGG_CUDA(cudaMemcpyAsync(h, prof, sizeof(h), cudaMemcpyDeviceToHost, ws.stream));
       EGG_CUDA(cudaStreamSynchronize(ws.stream));
       const double t = (double)(h[15] ? h[15] : 1);
-      fprintf(stderr, "[tc-prof] clk per entry tile: producer fetch %.0f (stage wait %.0f) wait_copies %.0f build %.0f | "
-              "classifier (per own tile) wait_S %.0f ld %.0f band %.0f wait_st %.0f | GEMM1 wait_full %.0f wait_free %.0f | "
-              "GEMM2 wait_P %.0f\n", h[4] / t, h[7] / t, h[5] / t, h[6] / t, h[0] / t, h[1] / t, h[2] / t, h[3] / t, h[8] / t,
-              h[9] / t, h[12] / t);
+      fprintf(stderr, "[tc-prof] clk per entry tile: copy warp issue %.0f (stage wait %.0f) | builders wait_landed %.0f "
+              "build %.0f | classifiers (per own tile) wait_S %.0f ld %.0f band %.0f wait_st %.0f | GEMM1 wait_full %.0f "
+              "wait_free %.0f | GEMM2 wait_P %.0f\n", h[10] / t, h[11] / t, h[4] / t, h[5] / t, h[0] / t, h[1] / t,
+              h[2] / t, h[3] / t, h[8] / t, h[9] / t, h[12] / t);
     }
 #endif
     if (ws.tc_timing) {
