@@ -262,9 +262,7 @@ int Workspace::alloc(int64_t n_, int d_, float eps, int dev, cudaStream_t st, do
       {(void**)&t_parent, sizeof(int32_t) * cap},
       {(void**)&l_parent, sizeof(int32_t) * cap},
       {(void**)&t_visit, sizeof(uint32_t) * cap},
-      {(void**)&t_fix, sizeof(uint64_t) * 2 * d * cap},
-      {(void**)&t_lo, sizeof(uint32_t) * d * cap},
-      {(void**)&t_hi, sizeof(uint32_t) * d * cap},
+      {(void**)&t_fix, sizeof(uint64_t) * 3 * d * cap},  // k_tree_agg rows: exact sums [2d], (hi<<32|lo) [d]
       {(void**)&t_cnt, sizeof(int32_t) * cap},
       {(void**)&t_box, sizeof(float) * BS * cap},
       {(void**)&t_sum, sizeof(float) * BS * cap},

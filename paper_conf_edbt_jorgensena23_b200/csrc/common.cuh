@@ -214,9 +214,7 @@ struct Workspace {
   int32_t* t_parent = nullptr; // [cap] parent of internal node
   int32_t* l_parent = nullptr; // [cap] parent of leaf (cell)
   uint32_t* t_visit = nullptr;
-  uint64_t* t_fix = nullptr;   // [2d][cap]
-  uint32_t* t_lo = nullptr;    // [d][cap]
-  uint32_t* t_hi = nullptr;
+  uint64_t* t_fix = nullptr;   // [cap][3d]: exact subtree sums [2d], (hi << 32 | lo) MBR bits [d]
   int32_t* t_cnt = nullptr;
   float* t_box = nullptr;      // [cap][2d] lo then hi
   float* t_sum = nullptr;      // [cap][2d] sin then cos

@@ -437,9 +437,11 @@ __global__ void k_tree_agg(int32_t nc, int64_t cap, const int4* __restrict__ met
                            const int32_t* __restrict__ t_parent, const int32_t* __restrict__ l_parent,
                            uint32_t* __restrict__ visit, const uint64_t* __restrict__ c_fix,
                            const uint32_t* __restrict__ c_lo, const uint32_t* __restrict__ c_hi,
-                           const int32_t* __restrict__ c_cnt, uint64_t* t_fix, uint32_t* t_lo,
-                           uint32_t* t_hi, int32_t* t_cnt, float* __restrict__ t_box,
-                           float* __restrict__ t_sum) {
+                           const int32_t* __restrict__ c_cnt, uint64_t* t_agg, int32_t* t_cnt,
+                           float* __restrict__ t_box, float* __restrict__ t_sum) {
+  // t_agg: one row of 3D u64 per internal node (exact sums [2D], then (hi << 32 | lo) [D]):
+  // a parent reads an internal child's exact aggregate from one contiguous row (cells keep
+  // their SoA c_fix / c_lo / c_hi)
   const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (c >= nc) return;
   constexpr int BS = ceil4(2 * D);
@@ -461,29 +463,38 @@ __global__ void k_tree_agg(int32_t nc, int64_t cap, const int4* __restrict__ met
     }
 #pragma unroll
     for (int k = 0; k < 2; ++k) {
-      const bool leaf = (ch[k] & (int32_t)kLeafBit) != 0;
       const int64_t x = ch[k] & 0x7fffffff;
-      const uint64_t* F = leaf ? c_fix : t_fix;
-      const uint32_t* L = leaf ? c_lo : t_lo;
-      const uint32_t* H = leaf ? c_hi : t_hi;
-      cnt += __ldcg(leaf ? &c_cnt[x] : &t_cnt[x]);
+      if (ch[k] & (int32_t)kLeafBit) {
+        cnt += __ldcg(&c_cnt[x]);
 #pragma unroll
-      for (int i = 0; i < 2 * D; ++i) fs[i] += __ldcg((const unsigned long long*)&F[(int64_t)i * cap + x]);
+        for (int i = 0; i < 2 * D; ++i) fs[i] += __ldcg((const unsigned long long*)&c_fix[(int64_t)i * cap + x]);
 #pragma unroll
-      for (int i = 0; i < D; ++i) {
-        lo[i] = min(lo[i], __ldcg(&L[(int64_t)i * cap + x]));
-        hi[i] = max(hi[i], __ldcg(&H[(int64_t)i * cap + x]));
+        for (int i = 0; i < D; ++i) {
+          lo[i] = min(lo[i], __ldcg(&c_lo[(int64_t)i * cap + x]));
+          hi[i] = max(hi[i], __ldcg(&c_hi[(int64_t)i * cap + x]));
+        }
+      } else {
+        cnt += __ldcg(&t_cnt[x]);
+        const unsigned long long* row = reinterpret_cast<const unsigned long long*>(t_agg + x * (3 * D));
+#pragma unroll
+        for (int i = 0; i < 2 * D; ++i) fs[i] += __ldcg(row + i);
+#pragma unroll
+        for (int i = 0; i < D; ++i) {
+          const unsigned long long b = __ldcg(row + 2 * D + i);
+          lo[i] = min(lo[i], (uint32_t)b);
+          hi[i] = max(hi[i], (uint32_t)(b >> 32));
+        }
       }
     }
+    uint64_t* row = t_agg + (int64_t)node * (3 * D);
 #pragma unroll
     for (int i = 0; i < 2 * D; ++i) {
-      t_fix[(int64_t)i * cap + node] = fs[i];
+      row[i] = fs[i];
       t_sum[(int64_t)node * BS + i] = (float)((double)(long long)fs[i] * kInvFix);
     }
 #pragma unroll
     for (int i = 0; i < D; ++i) {
-      t_lo[(int64_t)i * cap + node] = lo[i];
-      t_hi[(int64_t)i * cap + node] = hi[i];
+      row[2 * D + i] = ((uint64_t)hi[i] << 32) | lo[i];
       t_box[(int64_t)node * BS + i] = ord2f(lo[i]);
       t_box[(int64_t)node * BS + D + i] = ord2f(hi[i]);
     }
@@ -663,7 +674,7 @@ static int build_d(Workspace& ws) {
     EGG_LAUNCH_CHECK();
     k_tree_agg<D><<<blocks_for(nc, 128), 128, 0, st>>>(nc, cap, ws.t_meta, ws.t_parent, ws.l_parent,
                                                        ws.t_visit, ws.c_fix, ws.c_lo, ws.c_hi, ws.c_cnt,
-                                                       ws.t_fix, ws.t_lo, ws.t_hi, ws.t_cnt, ws.t_box,
+                                                       ws.t_fix, ws.t_cnt, ws.t_box,
                                                        ws.t_sum);
     EGG_LAUNCH_CHECK();
   }
