@@ -60,9 +60,12 @@ extern "C" {
 #define EGGSYNC_TERM_DEF42 1 /* Def 4.2 literally (L106-110): term (i) "no pair with eps/2 < ||p-q|| <= eps",
                                 term (ii) with MBR(N_{eps/2}(q)); labels = connected components of
                                 the eps-graph of the returned state (Theorem 4.7).  eggsync_cluster_ex
-                                only; runs on the direct (all-pairs, O(n^2 d) per iteration) kernels of
-                                eggsync_sync_step, not the grid, on opts.stream (NULL: the
-                                legacy default stream); ignores cw_factor and stats other
+                                only; the grid update, the terms and the labels evaluated on the
+                                grid's radix tree (work proportional to the neighbourhoods, F3). */
+#define EGGSYNC_TERM_DEF42_DIRECT 2 /* the same criterion and labels on the direct (all-pairs,
+                                O(n^2 d) per iteration) kernels of eggsync_sync_step, not the grid:
+                                a second implementation for cross-checks; on opts.stream (NULL:
+                                the legacy default stream); ignores cw_factor and stats other
                                 than iters. */
 
 /*
@@ -85,7 +88,7 @@ typedef struct eggsync_opts {
   int32_t device;          /* CUDA ordinal; -1 = current device */
   int32_t device_pointers; /* 1: points / labels / coords_out / nbr_count_out are device pointers */
   void *stream;            /* cudaStream_t to run on; NULL = library-owned stream */
-  int32_t term_mode;       /* EGGSYNC_TERM_GRID (default) or EGGSYNC_TERM_DEF42 (cluster_ex only) */
+  int32_t term_mode;       /* EGGSYNC_TERM_GRID (default), _DEF42 or _DEF42_DIRECT (cluster_ex only) */
   float *coords_out;       /* optional n*d row-major final coordinates (original point order) */
   int32_t *nbr_count_out;  /* optional, step only: |N_eps(p)| on D^t, original order */
   eggsync_stats *stats;    /* optional */

@@ -516,6 +516,51 @@ static int run_loop(Workspace& ws, int32_t max_iters, int32_t* iters_out, eggsyn
   return synced ? EGGSYNC_OK : EGGSYNC_NOT_CONVERGED;
 }
 
+// Algorithm 4 with Def 4.2 literally (term_mode = EGGSYNC_TERM_DEF42, F3): the same grid
+// update; term (i), MBR(N_{eps/2}) and term (ii) on the grid structure of D^t (def42_grid.cu);
+// labels = eps-graph components of the returned state (as the oracle's DEF42 mode).
+static int run_loop_def42(Workspace& ws, int32_t max_iters, int32_t* iters_out) {
+  struct Scratch {
+    void* p = nullptr;
+    ~Scratch() {
+      if (p) cudaFree(p);
+    }
+  } sc;
+  const size_t fb = sizeof(float) * (size_t)ws.n * ws.d;
+  EGG_CUDA(cudaMalloc(&sc.p, 2 * fb + 4 * sizeof(int32_t) * (size_t)ws.n));
+  float* mlo = reinterpret_cast<float*>(sc.p);
+  float* mhi = mlo + (size_t)ws.n * ws.d;
+  int32_t* lab_scratch = reinterpret_cast<int32_t*>(mhi + (size_t)ws.n * ws.d);
+  int32_t t = 0, synced = 0;
+  ws.have_final = false;
+  for (;;) {
+    if (!ws.built) EGG_TRY(stage_build(ws));
+    k_set_flags<<<1, 1, 0, ws.stream>>>(ws.flags, 1, 1);
+    EGG_CUDA(cudaGetLastError());
+    EGG_TRY(stage_update(ws, 0, ws.n, nullptr));
+    k_set_flags<<<1, 1, 0, ws.stream>>>(ws.flags, 1, 1);  // the update's grid first term is not used
+    EGG_CUDA(cudaGetLastError());
+    ws.launches += 2;
+    EGG_TRY(def42_grid_first(ws));
+    int32_t f1 = 0, f2 = 0;
+    EGG_TRY(read_flags(ws, &f1, nullptr, nullptr));
+    if (f1) {
+      EGG_TRY(def42_grid_second(ws, mlo, mhi));
+      EGG_TRY(read_flags(ws, nullptr, &f2, nullptr));
+    }
+    synced = f1 && f2;
+    advance(ws);
+    ++t;
+    if (synced || t >= max_iters) break;
+  }
+  EGG_TRY(stage_build(ws));  // the returned state D^t
+  EGG_TRY(def42_grid_labels(ws, lab_scratch, ws.lab_final));
+  ws.have_final = true;
+  EGG_CUDA(cudaStreamSynchronize(ws.stream));
+  *iters_out = t;
+  return synced ? EGGSYNC_OK : EGGSYNC_NOT_CONVERGED;
+}
+
 struct DeviceGuard {
   int prev = -1;
   bool changed = false;
@@ -617,8 +662,9 @@ static int get_opts(const eggsync_opts* in, eggsync_opts* o) {
     set_error("cw_factor=%g must be in (0, 1] (c_w <= eps/(2 sqrt d), L252)", o->cw_factor);
     return EGGSYNC_EINVAL;
   }
-  if (o->term_mode != EGGSYNC_TERM_GRID && o->term_mode != EGGSYNC_TERM_DEF42) {
-    set_error("term_mode %d unknown (EGGSYNC_TERM_GRID or EGGSYNC_TERM_DEF42)", o->term_mode);
+  if (o->term_mode != EGGSYNC_TERM_GRID && o->term_mode != EGGSYNC_TERM_DEF42 &&
+      o->term_mode != EGGSYNC_TERM_DEF42_DIRECT) {
+    set_error("term_mode %d unknown (EGGSYNC_TERM_GRID, _DEF42 or _DEF42_DIRECT)", o->term_mode);
     return EGGSYNC_EINVAL;
   }
   return EGGSYNC_OK;
@@ -711,8 +757,8 @@ int eggsync_cluster_ex(const float* points, int64_t n, int32_t d, float eps, con
   EGG_TRY(check_device());
   DeviceGuard g;
   EGG_TRY(g.set(o.device));
-  if (o.term_mode == EGGSYNC_TERM_DEF42) return def42_cluster(points, n, d, eps, o, labels_out, iters_out);
-  {
+  if (o.term_mode == EGGSYNC_TERM_DEF42_DIRECT) return def42_cluster(points, n, d, eps, o, labels_out, iters_out);
+  if (o.term_mode == EGGSYNC_TERM_GRID) {
     // F1: small inputs run Algorithm 4 in one kernel launch (no per-iteration host round trip);
     // validation of the domain happens inside (a point outside [0,1] is rejected below first)
     Consts kc;
@@ -741,7 +787,8 @@ int eggsync_cluster_ex(const float* points, int64_t n, int32_t d, float eps, con
   EGG_TRY(stage_ingest(ws, points, o.device_pointers != 0));
   auto t2 = std::chrono::steady_clock::now();
   int32_t iters = 0;
-  int rc = run_loop(ws, o.max_iters, &iters, stats);
+  int rc = o.term_mode == EGGSYNC_TERM_DEF42 ? run_loop_def42(ws, o.max_iters, &iters)
+                                              : run_loop(ws, o.max_iters, &iters, stats);
   if (rc < 0) return rc;
   // outputs
   auto t3 = std::chrono::steady_clock::now();

@@ -291,6 +291,11 @@ int stage_second_term(Workspace& ws, int64_t lo, int64_t hi);
 int stage_labels(Workspace& ws, int32_t* labels_dev);  // labels of current cells, original order
 int stage_coords(Workspace& ws, int which, float* out_dev);  // row-major, original order
 int stage_scatter_i32(Workspace& ws, const int32_t* sorted_vals, int32_t* out_dev);
+// F3, Def 4.2 on the grid structure (def42_grid.cu): term (i) into flags[0]; term (ii) into
+// flags[1] (mlo/mhi: [d][n] scratch); eps-graph labels of the built state (scratch: 4n int32)
+int def42_grid_first(Workspace& ws);
+int def42_grid_second(Workspace& ws, float* mlo, float* mhi);
+int def42_grid_labels(Workspace& ws, int32_t* scratch, int32_t* labels_dev);
 
 int tc_ranges_reserve(Workspace& ws, size_t need);  // grow ws.tc_ranges to >= need entries
 int tc_ent_reserve(Workspace& ws, size_t need);     // grow ws.tc_ent to >= need entries

@@ -139,6 +139,14 @@ struct WarpSmem {
   __host__ __device__ static size_t bytes(int stack_len) { return off_stk() + (size_t)stack_len * 16; }
 };
 
+// warps per update CTA: 4, fewer when 4 warps' shared memory at the deepest possible stack
+// (512 key bits) would exceed the 227 KB per CTA (d >= ~30)
+template <int D>
+struct UpdWarps {
+  static constexpr size_t kMax = WarpSmem<D>::off_stk() + (size_t)(64 * kMaxKeyWords + 4) * 16;
+  static constexpr int v = 4 * kMax <= 232448 ? 4 : 3 * kMax <= 232448 ? 3 : 2;
+};
+
 // ---- TMA (cp.async.bulk) staging of cell records: global -> shared, mbarrier completion
 __device__ __forceinline__ unsigned smem_u32(const void* p) {
   return static_cast<unsigned>(__cvta_generic_to_shared(p));
@@ -464,7 +472,7 @@ __device__ __forceinline__ void process_cells(const UpdArgs<D>& a, Lane<D>& L, i
 }
 
 template <int D, bool CNT>
-__global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(const UpdArgs<D> a) {
+__global__ void __launch_bounds__(UpdWarps<D>::v * 32, EGG_UPD_MINB) k_update(const UpdArgs<D> a) {
   constexpr int kP = PPL<D>::v;
   using W = WarpSmem<D>;
   constexpr int BS = ceil4(2 * D);
@@ -483,7 +491,7 @@ __global__ void __launch_bounds__(kWarpsPerCta * 32, EGG_UPD_MINB) k_update(cons
 
   // ownership blocks of kOwnBlock points (b % stride == offset), each split into warp blocks
   constexpr int kSub = kOwnBlock / (32 * kP);
-  const int64_t g = (int64_t)blockIdx.x * kWarpsPerCta + wid;
+  const int64_t g = (int64_t)blockIdx.x * UpdWarps<D>::v + wid;
   const int64_t base = a.lo + ((g / kSub) * a.stride + a.offset) * kOwnBlock + (g % kSub) * (32 * kP);
   Lane<D> L;
   unsigned long long amask = 0ull;
@@ -721,7 +729,7 @@ int run_update_simt(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   a.flags = ws.flags;
   a.nbr = nbr;
   a.work = ws.count_work ? ws.work : nullptr;
-  const size_t smem = (size_t)kWarpsPerCta * WarpSmem<D>::bytes(a.stack_len);
+  const size_t smem = (size_t)UpdWarps<D>::v * WarpSmem<D>::bytes(a.stack_len);
   auto kern = a.work ? k_update<D, true> : k_update<D, false>;
   EGG_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
   // all of the 228 KB unified L1/shared to shared memory: occupancy is shared-memory bound
@@ -733,8 +741,8 @@ int run_update_simt(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   const int64_t owned = nblocks > a.offset ? (nblocks - a.offset + a.stride - 1) / a.stride : 0;
   if (owned == 0) return EGGSYNC_OK;
   const int64_t warps = owned * (kOwnBlock / (32 * PPL<D>::v));
-  const unsigned grid = (unsigned)((warps + kWarpsPerCta - 1) / kWarpsPerCta);
-  kern<<<grid, kWarpsPerCta * 32, smem, ws.stream>>>(a);
+  const unsigned grid = (unsigned)((warps + UpdWarps<D>::v - 1) / UpdWarps<D>::v);
+  kern<<<grid, UpdWarps<D>::v * 32, smem, ws.stream>>>(a);
   ws.launches += 1;
   EGG_CUDA(cudaGetLastError());
   return EGGSYNC_OK;

@@ -163,7 +163,7 @@ def _host_points(points, writable=False):
     return a.copy() if writable else a  # step() writes D^{t+1}: never alias the caller's array
 
 
-TERM_GRID, TERM_DEF42 = 0, 1
+TERM_GRID, TERM_DEF42, TERM_DEF42_DIRECT = 0, 1, 2
 
 
 def cluster(points, eps: float, *, max_iters: int = 10000, coords: bool = False, stats: bool = False,

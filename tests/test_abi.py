@@ -128,12 +128,13 @@ def test_cw_factor_out_of_range_is_einval(f):
 
 
 def test_term_mode_validation():
-    """term_mode: GRID (0) or DEF42 (1, cluster_ex only); anything else EINVAL before any output."""
+    """term_mode: GRID (0), DEF42 (1) or DEF42_DIRECT (2), the last two cluster_ex only; anything
+    else EINVAL before any output."""
     pts = np.full((4, 2), 0.5, np.float32)
     lab = np.full(4, -7, np.int32)
     it = ctypes.c_int32(-9)
     o = E.default_opts()
-    o.term_mode = 2
+    o.term_mode = 3
     rc = E.lib().eggsync_cluster_ex(pts.ctypes.data_as(ctypes.c_void_p), 4, 2, ctypes.c_float(0.05),
                                     ctypes.byref(o), lab.ctypes.data_as(ctypes.c_void_p), ctypes.byref(it))
     assert rc == E.EINVAL and (lab == -7).all() and it.value == -9

@@ -107,7 +107,10 @@ def test_cluster_parity_c1(seed):
 
 @pytest.mark.parametrize("n,d,k,noise,eps,seed", [(4000, 3, 5, 0.0, 0.05, 0), (3000, 5, 10, 0.0, 0.05, 1),
                                                   (5000, 10, 20, 0.05, 0.1, 0), (2000, 20, 5, 0.0, 0.05, 2),
-                                                  (3333, 4, 3, 0.1, 0.07, 5), (1024, 32, 4, 0.0, 0.4, 1)])
+                                                  (3333, 4, 3, 0.1, 0.07, 5), (1024, 32, 4, 0.0, 0.4, 1),
+                                                  # d=32 at 6 key bits per dimension: 4 update warps
+                                                  # would need 234 KB of shared memory (UpdWarps)
+                                                  (1500, 32, 4, 0.0, 0.3, 2), (1200, 29, 3, 0.05, 0.2, 3)])
 def test_cluster_parity_shapes(n, d, k, noise, eps, seed):
     _cluster_compare(datagen.blobs(n, d, k, noise=noise, seed=seed), eps)
 
