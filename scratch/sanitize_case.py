@@ -14,4 +14,6 @@ elif case == "simt":
     os.environ["EGGSYNC_TC"] = "0"; r = E.cluster(datagen.blobs(20000, 10, 5, noise=0.05, seed=1), 0.25)
 elif case == "def42":
     r = E.cluster(datagen.blobs(3000, 3, 4, seed=2), 0.08, term_mode=E.TERM_DEF42)
+elif case == "def42_direct":
+    r = E.cluster(datagen.blobs(3000, 3, 4, seed=2), 0.08, term_mode=E.TERM_DEF42_DIRECT)
 print(case, "iters", r["iters"], "clusters", int(r["labels"].max()) + 1)
