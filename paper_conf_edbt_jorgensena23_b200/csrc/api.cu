@@ -191,6 +191,10 @@ int tc_ranges_reserve(Workspace& ws, size_t need) {
   return rc;
 }
 
+int dense_reserve(Workspace& ws, size_t cells) {
+  return buf_reserve(ws, 2, (void**)&ws.dense, &ws.dense_bytes, cells * sizeof(int32_t));
+}
+
 int tc_ent_reserve(Workspace& ws, size_t need) {
   size_t cb = ws.tc_ecap * sizeof(int32_t);
   const int rc = buf_reserve(ws, 1, (void**)&ws.tc_ent, &cb, need * sizeof(int32_t));
@@ -340,6 +344,9 @@ void Workspace::release() {
   }
   buf_give(cur_device, 0, tc_ranges, tc_rcap * sizeof(int2));
   buf_give(cur_device, 1, tc_ent, tc_ecap * sizeof(int32_t));
+  buf_give(cur_device, 2, dense, dense_bytes);
+  dense = nullptr;
+  dense_bytes = 0;
   tc_ent = nullptr;
   tc_ecap = 0;
   tc_ranges = nullptr;

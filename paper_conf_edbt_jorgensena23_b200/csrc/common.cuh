@@ -259,6 +259,8 @@ struct Workspace {
   size_t tc_ecap = 0;
   int32_t* tc_ctr = nullptr;    // [8] ranges allocated, chunk-table overflow, entries (u64), points in entries (u64), padded entries (u64)
   int32_t* tc_pv = nullptr;     // [tiles] tile index (sort values)
+  int32_t* dense = nullptr;     // F3 random-access grid: [w^d] grid cell per cell index (update_dense.cu)
+  size_t dense_bytes = 0;
   int32_t* tc_pk = nullptr;     // [tiles] entries, sorted descending (sort keys out)
   int32_t* tc_perm = nullptr;   // [tiles] launch order of the point tiles: most entries first
   int2* tc_ranges = nullptr;    // (first unit, count), grown on demand (process cache)
@@ -296,6 +298,11 @@ int stage_scatter_i32(Workspace& ws, const int32_t* sorted_vals, int32_t* out_de
 int def42_grid_first(Workspace& ws);
 int def42_grid_second(Workspace& ws, float* mlo, float* mhi);
 int def42_grid_labels(Workspace& ws, int32_t* scratch, int32_t* labels_dev);
+// F3, the random-access grid (§4.2.2) for d <= 4 (update_dense.cu)
+int64_t dense_cells(const Workspace& ws);
+bool dense_choose(const Workspace& ws);
+int dense_reserve(Workspace& ws, size_t cells);
+int run_update_dense(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr);
 
 int tc_ranges_reserve(Workspace& ws, size_t need);  // grow ws.tc_ranges to >= need entries
 int tc_ent_reserve(Workspace& ws, size_t need);     // grow ws.tc_ent to >= need entries

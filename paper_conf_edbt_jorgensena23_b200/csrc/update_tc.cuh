@@ -1413,6 +1413,9 @@ inline bool tc_enabled(const Workspace& ws, int d) {
 template <int D>
 int run_update(Workspace& ws, int64_t lo, int64_t hi, int32_t* nbr) {
   ws.tc_used = 0;
+  if constexpr (D <= 4) {  // F3 random-access grid when selected (single-process updates)
+    if (ws.tc_mode == 0 && dense_choose(ws)) return run_update_dense(ws, lo, hi, nbr);
+  }
   if (tc_enabled(ws, D) && hi > lo) return run_update_tc<D>(ws, lo, hi, nbr);
   if (ws.tc_mode == 1) {  // plan only, tensor cores off on every rank (replicated cell count)
     for (auto& v : ws.tc_local) v = 0;
