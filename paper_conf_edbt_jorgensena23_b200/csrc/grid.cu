@@ -447,8 +447,11 @@ __global__ void k_tree_agg(int32_t nc, int64_t cap, const int4* __restrict__ met
   constexpr int BS = ceil4(2 * D);
   int32_t node = l_parent[c];
   while (node >= 0) {
-    __threadfence();
-    if (atomicAdd(&visit[node], 1u) == 0u) return;  // first arrival: sibling not ready
+    // acq_rel: the first arrival releases its subtree's aggregate (written by this thread the
+    // level below), the second acquires the sibling's before reading it (no full fence)
+    uint32_t prev;
+    asm volatile("atom.acq_rel.gpu.global.add.u32 %0, [%1], 1;" : "=r"(prev) : "l"(&visit[node]) : "memory");
+    if (prev == 0u) return;  // first arrival: sibling not ready
     const int4 m = meta[node];
     const int32_t ch[2] = {m.z, m.w};
     uint64_t fs[2 * D];
