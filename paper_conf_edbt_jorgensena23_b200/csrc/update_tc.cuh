@@ -34,9 +34,9 @@
 //   warps 8-11  builders: thread t owns entry slot t; from the landed record head it writes the
 //               origin-shifted, fp16-split GEMM1 operand row and the band width
 //   warp 12     MMA issue (one thread issues GEMM1 and GEMM2 in tile order) and TMEM owner
-//   warps 13-15 copy warps: fill the ring stages (up to 8) with per-lane cp.async, each warp
-//               every third entry tile, up to NST tiles ahead (the gathers by unit index are
-//               latency-bound per warp)
+//   warps 13-15 copy warps: fill the ring stages (up to 8) with per-thread cp.async, all three
+//               on every entry tile (slots t, t + 96), up to NST tiles ahead (the gathers by unit
+//               index are latency-bound per warp)
 // Waiting warps poll one per group and park the others in a named barrier.
 // TMEM: Q (K1 columns) | 2-3 S/P buffers of 128 columns | O (N columns, int32).
 #pragma once
@@ -694,7 +694,7 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
   // ---- setup -------------------------------------------------------------------------
   if (tid == 0) {
     for (int s = 0; s < NST; ++s) {
-      tc::bar_init(&ms->stage_landed[s], 32);    // one cp.async-completion arrival per copy lane
+      tc::bar_init(&ms->stage_landed[s], 32 * kCopyWarps);  // one cp.async-completion arrival per copy thread
       tc::bar_init(&ms->stage_full[s], kProd);   // one arrival per builder thread (entry slot)
       tc::bar_init(&ms->stage_empty[s], 1);
     }
@@ -836,45 +836,48 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
 
   if (wid >= kCopyWarp0) {
     // ================================ copy warps ================================
-    // Copy warp w fills the stages of entry tiles t = w mod kCopyWarps (several warps: the
-    // gathers by unit index are latency-bound per warp), up to NST tiles ahead: the tile's 128
-    // slot units (512 B of the slot list) and, for slot e = lane + 32 j, its record head and
-    // digit row by 16-byte cp.async (block-major global layouts: consecutive lanes read
-    // consecutive units of a run, so the copies coalesce).  Each lane's completion arrives on
-    // stage_landed (cp.async.mbarrier.arrive.noinc); the warps never wait for their copies.
+    // The copy warps (96 threads) fill the stage of every entry tile together, up to NST tiles
+    // ahead: thread t copies slots t and t + 96 -- the slot's unit (slot list), its record head
+    // and its digit row, by 16-byte cp.async (block-major global layouts: consecutive threads
+    // read consecutive units of a run, so the copies coalesce) -- and the tile's 512 B of slot
+    // units come from threads 0..31.  Splitting every tile over all copy threads keeps the time
+    // from a stage's release to its refill short (the gathers are latency-bound per warp).
+    // Each thread's completion arrives on stage_landed (cp.async.mbarrier.arrive.noinc).
     constexpr int NH = R0 / 4;
+    constexpr int kCT = 32 * kCopyWarps;  // copy threads
     const int nchunk = N2 / 16;
-    const int cw = wid - kCopyWarp0;
+    const int ct = tid - 32 * kCopyWarp0;
     const int32_t* __restrict__ ent = a.ent + a.eoff[tile];  // 512-byte aligned (padded tiles)
     const char* __restrict__ hb = reinterpret_cast<const char*>(a.c_head);
     const char* __restrict__ db = reinterpret_cast<const char*>(a.c_dig);
     const int64_t capB = a.cap * 16;  // bytes of one 16-byte block column
-    int cn[4];
+    constexpr int kSl = (kTcEnt + kCT - 1) / kCT;  // slots per copy thread
+    int cn[kSl];
 #pragma unroll
-    for (int j = 0; j < 4; ++j) cn[j] = cw < T ? ent[(int64_t)cw * kTcEnt + lane + 32 * j] : -1;
+    for (int j = 0; j < kSl; ++j) cn[j] = (T > 0 && ct + kCT * j < kTcEnt) ? ent[ct + kCT * j] : -1;
     RingPos fp;
-    for (int k = 0; k < cw; ++k) fp.adv(NST);
-    for (int t = cw; t < T; t += kCopyWarps) {
-      int cu[4];
+    for (int t = 0; t < T; ++t) {
+      int cu[kSl];
 #pragma unroll
-      for (int j = 0; j < 4; ++j) cu[j] = cn[j];
-      if (t + kCopyWarps < T) {
+      for (int j = 0; j < kSl; ++j) cu[j] = cn[j];
+      if (t + 1 < T) {
 #pragma unroll
-        for (int j = 0; j < 4; ++j) cn[j] = ent[(int64_t)(t + kCopyWarps) * kTcEnt + lane + 32 * j];
+        for (int j = 0; j < kSl; ++j)
+          cn[j] = ct + kCT * j < kTcEnt ? ent[(int64_t)(t + 1) * kTcEnt + ct + kCT * j] : -1;
       }
       TCP_T(f0);
       if (t >= NST) {
-        if (lane == 0) tc::bar_poll(&ms->stage_empty[fp.i], fp.ph ^ 1u);
-        __syncwarp();
+        if (ct == 0) tc::bar_poll(&ms->stage_empty[fp.i], fp.ph ^ 1u);
+        tc::named_sync(4, kCT);
       }
       TCP_T(f1);
       TcStage<D> st(ring, fp.i, SB, N2);
-      cp_async16(st.cell + 4 * lane, ent + (int64_t)t * kTcEnt + 4 * lane);
+      if (ct < 32) cp_async16(st.cell + 4 * ct, ent + (int64_t)t * kTcEnt + 4 * ct);
 #pragma unroll
-      for (int j = 0; j < 4; ++j) {
+      for (int j = 0; j < kSl; ++j) {
         const int c = cu[j];
         if (c >= 0) {
-          const int e = lane + 32 * j;
+          const int e = ct + kCT * j;
           const char* hs = hb + (int64_t)c * 16;
 #pragma unroll
           for (int k = 0; k < NH; ++k) cp_async16(st.rec + ((size_t)k * kTcEnt + e) * 4, hs + k * capB);
@@ -887,13 +890,10 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
       }
       asm volatile("cp.async.mbarrier.arrive.noinc.shared::cta.b64 [%0];" ::"r"(tc::smem_addr(&ms->stage_landed[fp.i]))
                    : "memory");
-#pragma unroll
-      for (int k = 0; k < kCopyWarps; ++k) fp.adv(NST);
+      fp.adv(NST);
       TCP_T(f2);
-      if (cw == 0) {
-        TCP_ADD(0, f2 - f1);
-        TCP_ADD(1, f1 - f0);
-      }
+      TCP_ADD(0, f2 - f1);
+      TCP_ADD(1, f1 - f0);
     }
     cp_async_wait<0>();
   }
@@ -1055,7 +1055,7 @@ __global__ void __launch_bounds__((kTcThreads + 127) / 128 * 128, 1) k_update_tc
     int slot = -1;
     if (tid == 0 || tid == 128) slot = 0;
     else if (tid == 256) slot = 4;
-    else if (wid == kCopyWarp0 && lane == 0) slot = 10;
+    else if (tid == 32 * kCopyWarp0) slot = 10;
     if (slot >= 0 && a.prof) {
       const int nk = slot == 12 ? 1 : slot == 0 ? 4 : 2;
       for (int k = 0; k < nk; ++k) atomicAdd(&a.prof[slot + k], prof_acc[k]);
