@@ -15,6 +15,7 @@ import numpy as np
 import pytest
 
 import oracle
+from tests import theorem47
 from paper_conf_edbt_jorgensena23_b200 import datagen
 from paper_conf_edbt_jorgensena23_b200 import eggsync as E
 
@@ -205,6 +206,13 @@ def test_c3_cluster_terminal_property(c3):
     assert np.array_equal(np.sort(first), first)  # canonical: ids by first occurrence
     idx = np.random.default_rng(1).choice(len(X), 64, replace=False)
     assert oracle.terminal_violations(r["coords"], c.eps, lab, idx) == 0
+    # the complete Theorem 4.7 property over all n (tests/theorem47.py: independent of the
+    # CUDA path and of the oracle): same label <=> within eps, for every pair
+    assert theorem47.violations(r["coords"], lab, c.eps) == 0
+    # Def 4.2 evaluated literally (term_mode DEF42, another criterion and another labelling:
+    # eps-graph components) reaches the same partition (Theorem 4.7), in no more iterations
+    d42 = E.cluster(X, c.eps, term_mode=E.TERM_DEF42)
+    assert d42["converged"] and np.array_equal(d42["labels"], lab) and d42["iters"] <= r["iters"]
 
 
 # ------------------------------------------------------------ full-size (C5, one GPU)
